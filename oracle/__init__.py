@@ -170,3 +170,15 @@ def sumsq(x) -> float:
 def energy(ext, t3, eps_h, eps_p) -> float:
     e = _ext(ext)
     return float(lib().oracle_energy(_p(e), _p(_c(t3)), _p(_c(eps_h)), _p(_c(eps_p))))
+
+
+def ccsdt_abs_bound(family: str, ext, t3, t2s, v2s) -> np.ndarray:
+    """Componentwise scale for tolerances (R14): |t3| + sum_v |t2_v|.|v2_v| sums,
+    i.e. the same contraction evaluated on absolute values with all signs positive."""
+    out = np.abs(_c(t3)).copy()
+    z = np.zeros_like(out)
+    for v in range(1, 10):
+        if t2s[v - 1] is None:
+            continue
+        out += np.abs(ccsdt(family, v, ext, z, np.abs(t2s[v - 1]), np.abs(v2s[v - 1])))
+    return out

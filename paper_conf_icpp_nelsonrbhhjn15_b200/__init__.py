@@ -1,0 +1,212 @@
+"""libbarracuda Python binding: B200-native batched small tensor contractions.
+
+Thin argument marshalling over the C ABI in include/barracuda.h (ctypes): every function
+checks dtype / device / contiguity / shape, then passes `data_ptr()`s and the current CUDA
+stream to the library.  All arithmetic happens in the sm_100a kernels; there is no CPU or
+PyTorch fallback (importing raises if libbarracuda.so is missing, and every call raises
+BarracudaError on a non-zero status).
+
+Method: Nelson et al., "Generating Efficient Tensor Contractions for GPUs", ICPP 2015
+ — see DESIGN.md for the path, the readings of the paper, and the layouts.
+"""
+from __future__ import annotations
+
+import ctypes
+from typing import Optional, Sequence
+
+import torch
+
+from . import _abi
+from ._abi import BC_CHECK_WS_DOUBLES, TileDims, lib
+
+__all__ = [
+    "BarracudaError", "sumfact3d", "sumfact2d", "local_grad3", "local_grad3_t", "ax_e",
+    "ccsdt", "ccsdt_fused", "check_sumsq", "check_energy", "fill", "launch_count",
+    "reset_launch_count", "LIB_PATH",
+]
+
+LIB_PATH = _abi.LIB_PATH
+
+
+class BarracudaError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        msg = lib.bc_status_string(status).decode()
+        if status == -5:
+            msg += f" (cudaError {lib.bc_last_cuda_error()})"
+        super().__init__(f"{where}: {msg}")
+        self.status = status
+
+
+def _check(status: int, where: str) -> None:
+    if status != 0:
+        raise BarracudaError(status, where)
+
+
+def _stream(t: torch.Tensor) -> ctypes.c_void_p:
+    return ctypes.c_void_p(torch.cuda.current_stream(t.device).cuda_stream)
+
+
+def _dev(t: torch.Tensor, dtype: torch.dtype, name: str) -> int:
+    if not isinstance(t, torch.Tensor):
+        raise TypeError(f"{name} must be a torch.Tensor")
+    if not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA tensor (no CPU path)")
+    if t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    return t.data_ptr()
+
+
+def _p_of(op: torch.Tensor, name: str) -> int:
+    if op.dim() != 2 or op.shape[0] != op.shape[1]:
+        raise ValueError(f"{name} must be square (p+1)x(p+1)")
+    return op.shape[0] - 1
+
+
+def _field(U: torch.Tensor, P1: int, ndim: int, name: str) -> int:
+    if U.dim() != ndim + 1 or tuple(U.shape[1:]) != (P1,) * ndim:
+        raise ValueError(f"{name} must have shape (N,{','.join(['p+1'] * ndim)}) with p+1={P1}")
+    return U.shape[0]
+
+
+# ----------------------------------------------------------------------------- spectral
+
+def sumfact3d(A, B, C, U, out: Optional[torch.Tensor] = None) -> torch.Tensor:
+    """V[e][i][j][k] = sum_lmn A[k][n] B[j][m] C[i][l] U[e][l][m][n]  (fp64 or fp32)."""
+    p = _p_of(A, "A")
+    N = _field(U, p + 1, 3, "U")
+    V = torch.empty_like(U) if out is None else out
+    dt = U.dtype
+    fn = {torch.float64: lib.bc_sumfact3d, torch.float32: lib.bc_sumfact3d_f32}.get(dt)
+    if fn is None:
+        raise TypeError("sumfact3d supports float64 and float32")
+    _check(fn(N, p, _dev(A, dt, "A"), _dev(B, dt, "B"), _dev(C, dt, "C"), _dev(U, dt, "U"),
+              _dev(V, dt, "out"), _stream(U)), "bc_sumfact3d")
+    return V
+
+
+def sumfact2d(A, B, U, out=None) -> torch.Tensor:
+    """V[e][i][j] = sum_lm B[i][l] A[j][m] U[e][l][m]  (V = B U A^T)."""
+    p = _p_of(A, "A")
+    N = _field(U, p + 1, 2, "U")
+    V = torch.empty_like(U) if out is None else out
+    f = torch.float64
+    _check(lib.bc_sumfact2d(N, p, _dev(A, f, "A"), _dev(B, f, "B"), _dev(U, f, "U"), _dev(V, f, "out"),
+                            _stream(U)), "bc_sumfact2d")
+    return V
+
+
+def local_grad3(D, U, out=None):
+    """(ur, us, ut) of Nekbone local_grad3 on U[e][k][j][i]."""
+    p = _p_of(D, "D")
+    N = _field(U, p + 1, 3, "U")
+    ur, us, ut = (torch.empty_like(U) for _ in range(3)) if out is None else out
+    f = torch.float64
+    _check(lib.bc_local_grad3(N, p, _dev(D, f, "D"), _dev(U, f, "U"), _dev(ur, f, "ur"), _dev(us, f, "us"),
+                              _dev(ut, f, "ut"), _stream(U)), "bc_local_grad3")
+    return ur, us, ut
+
+
+def local_grad3_t(D, ur, us, ut, out=None) -> torch.Tensor:
+    p = _p_of(D, "D")
+    N = _field(ur, p + 1, 3, "ur")
+    U = torch.empty_like(ur) if out is None else out
+    f = torch.float64
+    _check(lib.bc_local_grad3_t(N, p, _dev(D, f, "D"), _dev(ur, f, "ur"), _dev(us, f, "us"), _dev(ut, f, "ut"),
+                                _dev(U, f, "out"), _stream(ur)), "bc_local_grad3_t")
+    return U
+
+
+def ax_e(D, U, G, out=None) -> torch.Tensor:
+    """Nekbone element operator; G has shape (N, 6, p+1, p+1, p+1)."""
+    p = _p_of(D, "D")
+    N = _field(U, p + 1, 3, "U")
+    if tuple(G.shape) != (N, 6) + tuple(U.shape[1:]):
+        raise ValueError("G must have shape (N, 6, p+1, p+1, p+1)")
+    W = torch.empty_like(U) if out is None else out
+    f = torch.float64
+    _check(lib.bc_ax_e(N, p, _dev(D, f, "D"), _dev(U, f, "U"), _dev(G, f, "G"), _dev(W, f, "out"), _stream(U)),
+           "bc_ax_e")
+    return W
+
+
+# ----------------------------------------------------------------------------- CCSD(T)
+
+def _dims(ext: Sequence[int]) -> TileDims:
+    if len(ext) != 7:
+        raise ValueError("ext = (h1, h2, h3, p4, p5, p6, k)")
+    return TileDims(*[int(x) for x in ext])
+
+
+def ccsdt(family: str, variant: int, ext, t3: torch.Tensor, t2: torch.Tensor, v2: torch.Tensor) -> torch.Tensor:
+    """t3 += s_v * contraction of NWChem sd_t_<family>_<variant> (in place; returns t3).
+    family in {'d1','d2','s1'}; ext = (h1,h2,h3,p4,p5,p6,k); flat Fortran-ordered tensors."""
+    fn = {"d1": lib.bc_ccsdt_d1, "d2": lib.bc_ccsdt_d2, "s1": lib.bc_ccsdt_s1}[family]
+    f = torch.float64
+    d = _dims(ext)
+    _check(fn(int(variant), ctypes.byref(d), _dev(t3, f, "t3"), _dev(t2, f, "t2"), _dev(v2, f, "v2"),
+              _stream(t3)), f"bc_ccsdt_{family}")
+    return t3
+
+
+def ccsdt_fused(family: str, ext, t3: torch.Tensor, t2s, v2s) -> torch.Tensor:
+    """t3 += sum over v with t2s[v-1] not None (in place; returns t3)."""
+    fn = {"d1": lib.bc_ccsdt_d1_fused, "d2": lib.bc_ccsdt_d2_fused, "s1": lib.bc_ccsdt_s1_fused}[family]
+    f = torch.float64
+    a, b = _abi.PtrArray9(), _abi.PtrArray9()
+    for v in range(9):
+        if t2s[v] is not None:
+            a[v] = _dev(t2s[v], f, f"t2[{v}]")
+            b[v] = _dev(v2s[v], f, f"v2[{v}]")
+    d = _dims(ext)
+    _check(fn(ctypes.byref(d), _dev(t3, f, "t3"), a, b, _stream(t3)), f"bc_ccsdt_{family}_fused")
+    return t3
+
+
+# ----------------------------------------------------------------------------- checks
+
+def check_sumsq(x: torch.Tensor, ws: Optional[torch.Tensor] = None) -> torch.Tensor:
+    """Device scalar sum(x^2) (returned as a 0-d view of the workspace)."""
+    if ws is None:
+        ws = torch.empty(BC_CHECK_WS_DOUBLES, dtype=torch.float64, device=x.device)
+    f = torch.float64
+    _check(lib.bc_check_sumsq(x.numel(), _dev(x, f, "x"), _dev(ws, f, "ws"), _stream(x)), "bc_check_sumsq")
+    return ws[0]
+
+
+def check_energy(ext, t3, eps_h, eps_p, ws=None) -> torch.Tensor:
+    if ws is None:
+        ws = torch.empty(BC_CHECK_WS_DOUBLES, dtype=torch.float64, device=t3.device)
+    f = torch.float64
+    d = _dims(list(ext[:6]) + [1])
+    _check(lib.bc_check_energy(ctypes.byref(d), _dev(t3, f, "t3"), _dev(eps_h, f, "eps_h"), _dev(eps_p, f, "eps_p"),
+                               _dev(ws, f, "ws"), _stream(t3)), "bc_check_energy")
+    return ws[0]
+
+
+# ----------------------------------------------------------------------------- inputs
+
+KIND_REAL, KIND_INT, KIND_RANGE = 0, 1, 2
+
+
+def fill(out: torch.Tensor, tensor_id: int, kind: int = KIND_REAL, seed: int = 2015, offset: int = 0,
+         lo: float = -1.0, hi: float = 1.0) -> torch.Tensor:
+    """Counter-based synthetic values in place (same definition as synthetic/)."""
+    if out.dtype == torch.float64:
+        fn = lib.bc_fill
+    elif out.dtype == torch.float32:
+        fn = lib.bc_fill_f32
+    else:
+        raise TypeError("fill: float64 or float32")
+    _check(fn(int(kind), int(seed), int(tensor_id), int(offset), out.numel(), float(lo), float(hi),
+              _dev(out, out.dtype, "out"), _stream(out)), "bc_fill")
+    return out
+
+
+def launch_count() -> int:
+    return int(lib.bc_launch_count())
+
+
+def reset_launch_count() -> None:
+    lib.bc_reset_launch_count()

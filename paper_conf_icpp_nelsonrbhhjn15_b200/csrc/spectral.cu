@@ -1,0 +1,581 @@
+// Spectral-element family on sm_100a: sumfact3d (fp64/fp32), sumfact2d, local_grad3,
+// local_grad3_t and the fused Nekbone element operator ax_e.
+//
+// Design.  A CTA owns a group of E consecutive elements.  The group is
+// staged global -> shared memory with cp.async (LDGSTS) into a row-padded layout whose
+// strided row reads are bank-conflict free, prefetching the next group while the current
+// one computes.  Each contraction stage applies one (p+1)x(p+1) operator along one axis of
+// every element ("lines": P1 values along the contracted axis, held in registers).  A
+// thread owns R lines and accumulates each output in a register (the paper's scalar
+// replacement); operator rows are read as 16-byte broadcast pairs, so every
+// shared-memory wavefront feeds 2R FMAs.  Intermediates never leave shared memory
+// (fusion); only U in and the outputs touch HBM.
+#include <algorithm>
+
+#include "common.cuh"
+
+namespace bc {
+
+// ------------------------------------------------------------------------------------
+// Shared-memory geometry of one element: NA planes x P1 rows x RS (row stride).
+//  fp64: odd P1 -> RS = P1 (row stride odd: LDS.64 conflict-free);
+//        P1 = 2 mod 4 -> RS = P1 (RS/2 odd: 16-byte row reads conflict-free);
+//        P1 = 0 mod 4 -> RS = P1 + 2 (restores RS/2 odd).
+//  fp32: RS = P1 | 1 (odd stride, scalar row reads conflict-free).
+// ------------------------------------------------------------------------------------
+template <int P1, int NA, typename T>
+struct Geo {
+    static constexpr int RS = sizeof(T) == 8 ? ((P1 % 2) ? P1 : (((P1 / 2) % 2) ? P1 : P1 + 2))
+                                             : (P1 | 1);
+    static constexpr int PS = P1 * RS;          // plane stride in smem
+    static constexpr int ES = NA * PS;          // element stride in smem
+    static constexpr int NPTS = NA * P1 * P1;   // points per element in global memory
+    static constexpr int OS = (P1 + 1) & ~1;    // operator row stride (pairs aligned)
+    static constexpr bool PADDED = (RS != P1);
+    static constexpr bool VEC_ROWS = (sizeof(T) == 8) && (RS % 2 == 0);
+};
+
+// Stage `ne` elements (contiguous in global from `src`) into padded smem `dst`.
+template <int P1, int NA, typename T, int NT>
+__device__ __forceinline__ void load_group_async(T* __restrict__ dst, const T* __restrict__ src,
+                                                 int ne) {
+    using G = Geo<P1, NA, T>;
+    const int total = ne * G::NPTS;
+    if constexpr (!G::PADDED) {
+        // smem layout == global layout: 16-byte chunks when aligned
+        constexpr int V = 16 / sizeof(T);
+        const bool aligned = ((reinterpret_cast<uintptr_t>(src) & 15) == 0);
+        if (aligned) {
+            const int nvec = total / V;
+            for (int i = threadIdx.x; i < nvec; i += NT) cp_async_16(dst + i * V, src + i * V);
+            for (int i = nvec * V + threadIdx.x; i < total; i += NT) cp_async_elem(dst + i, src + i);
+        } else {
+            for (int i = threadIdx.x; i < total; i += NT) cp_async_elem(dst + i, src + i);
+        }
+    } else {
+        for (int f = threadIdx.x; f < total; f += NT) {
+            const int e = f / G::NPTS;
+            const int r = f - e * G::NPTS;  // (a, b, c) flattened
+            const int row = r / P1;         // (a, b)
+            const int c = r - row * P1;
+            cp_async_elem(dst + e * G::ES + row * G::RS + c, src + f);
+        }
+    }
+}
+
+// smem offset of global point f (element-relative flattened (e, a, b, c))
+template <int P1, int NA, typename T>
+__device__ __forceinline__ int smem_index(int f) {
+    using G = Geo<P1, NA, T>;
+    if constexpr (!G::PADDED) {
+        return f;
+    } else {
+        const int e = f / G::NPTS;
+        const int r = f - e * G::NPTS;
+        const int row = r / P1;
+        return e * G::ES + row * G::RS + (r - row * P1);
+    }
+}
+
+// First smem offset and stride of line L (element-relative) along AXIS.
+//   AXIS 2 (fastest, c): L = (e, a, b) -> rows;   AXIS 1 (b): L = (e, a, c);
+//   AXIS 0 (a, slowest): L = (e, b, c)  (only when NA == P1).
+template <int P1, int NA, int AXIS, typename T>
+struct Line {
+    using G = Geo<P1, NA, T>;
+    static constexpr int STRIDE = AXIS == 2 ? 1 : (AXIS == 1 ? G::RS : G::PS);
+    static constexpr int PER_ELEM = NA * P1;  // lines per element along any axis (NA*P1*P1/P1)
+    __device__ __forceinline__ static int base(int L) {
+        if constexpr (AXIS == 2) {
+            return L * G::RS;
+        } else if constexpr (AXIS == 1) {
+            const int e = L / (NA * P1);
+            const int r = L - e * (NA * P1);
+            const int a = r / P1;
+            return e * G::ES + a * G::PS + (r - a * P1);
+        } else {
+            const int e = L / (P1 * P1);
+            const int r = L - e * (P1 * P1);
+            const int b = r / P1;
+            return e * G::ES + b * G::RS + (r - b * P1);
+        }
+    }
+    // global (unpadded, element-relative) offset of output k of line L
+    __device__ __forceinline__ static int gofs(int L, int k) {
+        if constexpr (AXIS == 2) {
+            return L * P1 + k;
+        } else if constexpr (AXIS == 1) {
+            const int e = L / (NA * P1);
+            const int r = L - e * (NA * P1);
+            const int a = r / P1;
+            return e * G::NPTS + a * P1 * P1 + k * P1 + (r - a * P1);
+        } else {
+            const int e = L / (P1 * P1);
+            return e * G::NPTS + k * P1 * P1 + (L - e * (P1 * P1));
+        }
+    }
+};
+
+// out(L, base, k, value): consumer of one output value.
+// Applies op (P1 x P1 in smem, row stride OS) along AXIS of the lines [0, nlines):
+//     y(L, k) = sum_{n=0..P1-1} op[k][n] * x(L, n)       (ascending n)
+template <int P1, int NA, int AXIS, int R, int NT, typename T, typename Out>
+__device__ __forceinline__ void apply_lines(const T* __restrict__ in, const T* __restrict__ op,
+                                            int nlines, Out out) {
+    using G = Geo<P1, NA, T>;
+    using LN = Line<P1, NA, AXIS, T>;
+    using P2 = typename Pair<T>::type;
+    for (int L0 = threadIdx.x; L0 < nlines; L0 += R * NT) {
+        T x[R][P1];
+        int base[R];
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            int L = L0 + r * NT;
+            L = (L < nlines) ? L : L0;
+            base[r] = LN::base(L);
+            if constexpr (AXIS == 2 && G::VEC_ROWS) {
+#pragma unroll
+                for (int n = 0; n < P1; n += 2) {
+                    const P2 v = *reinterpret_cast<const P2*>(in + base[r] + n);
+                    x[r][n] = v.x;
+                    x[r][n + 1] = v.y;
+                }
+            } else {
+#pragma unroll
+                for (int n = 0; n < P1; ++n) x[r][n] = in[base[r] + n * LN::STRIDE];
+            }
+        }
+#pragma unroll 1
+        for (int k = 0; k < P1; ++k) {  // not unrolled: keeps only the lines in registers
+            T acc[R];
+#pragma unroll
+            for (int r = 0; r < R; ++r) acc[r] = T(0);
+#pragma unroll
+            for (int n = 0; n + 1 < P1; n += 2) {
+                const P2 o = *reinterpret_cast<const P2*>(op + k * G::OS + n);
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    acc[r] = fma(o.x, x[r][n], acc[r]);
+                    acc[r] = fma(o.y, x[r][n + 1], acc[r]);
+                }
+            }
+            if constexpr (P1 & 1) {
+                const T o = op[k * G::OS + P1 - 1];
+#pragma unroll
+                for (int r = 0; r < R; ++r) acc[r] = fma(o, x[r][P1 - 1], acc[r]);
+            }
+#pragma unroll
+            for (int r = 0; r < R; ++r)
+                if (L0 + r * NT < nlines) out(L0 + r * NT, base[r], k, acc[r]);
+        }
+    }
+}
+
+// operator staging: op_s[k][n] = M[k][n] (TRANSPOSE = false) or M[n][k] (true)
+template <int P1, typename T, int NT, bool TRANSPOSE = false>
+__device__ __forceinline__ void load_op(T* __restrict__ op_s, const T* __restrict__ M) {
+    constexpr int OS = (P1 + 1) & ~1;
+    for (int i = threadIdx.x; i < P1 * OS; i += NT) {
+        const int k = i / OS, n = i - (i / OS) * OS;
+        op_s[i] = (n < P1) ? (TRANSPOSE ? M[n * P1 + k] : M[k * P1 + n]) : T(0);
+    }
+}
+
+template <int P1, typename T>
+constexpr int op_elems() {  // rounded so that what follows stays 16-byte aligned
+    return (P1 * ((P1 + 1) & ~1) + (16 / (int)sizeof(T)) - 1) / (16 / (int)sizeof(T)) * (16 / (int)sizeof(T));
+}
+
+__host__ __device__ __forceinline__ int imin64(int64_t a, int64_t b) { return (int)(a < b ? a : b); }
+
+// ---------------------------------------------------------------- launch configuration
+// The fixed variant table (north star: "settled by ncu measurement and recorded in a
+// small fixed table"): elements per CTA E, threads NT, lines per thread R.
+template <int P1, int NA, typename T, int NBUF>
+struct Cfg {
+    using G = Geo<P1, NA, T>;
+    static constexpr int BUF_BYTES = 36 * 1024;  // per element-group buffer
+    static constexpr int E0 = BUF_BYTES / (G::ES * (int)sizeof(T));
+    static constexpr int E = E0 < 2 ? 1 : (E0 & ~1);  // even: groups of odd-P1 elements stay 16B-aligned
+    static constexpr int R = 2;
+    static constexpr int LINES = E * NA * P1;  // lines per axis per group (E * NPTS / P1)
+    static constexpr int NT0 = ((LINES + R - 1) / R + 31) / 32 * 32;
+    static constexpr int NT = NT0 < 64 ? 64 : (NT0 > 512 ? 512 : NT0);
+    static constexpr int BUF = (E * G::ES + (16 / (int)sizeof(T)) - 1) / (16 / (int)sizeof(T)) * (16 / (int)sizeof(T));
+    static constexpr size_t SMEM = (size_t)NBUF * BUF * sizeof(T) + 4 * op_elems<P1, T>() * sizeof(T);
+};
+
+template <typename KernelT>
+int grid_for(KernelT kernel, int nt, size_t smem, int64_t ngroups, int* occ_cache) {
+    if (*occ_cache == 0) {
+        cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        int occ = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, nt, smem);
+        *occ_cache = occ < 1 ? 1 : occ;
+    }
+    const int64_t cap = (int64_t)num_sms() * *occ_cache;
+    return imin64(ngroups, cap);
+}
+
+// ====================================================================== sumfact3d
+//   S1 W1[l][m][k] = sum_n A[k][n] U[l][m][n]     (axis 2, P:440 / Fig. 2(b))
+//   S2 W2[l][j][k] = sum_m B[j][m] W1[l][m][k]    (axis 1, P:441 / P:214)
+//   S3 V [i][j][k] = sum_l C[i][l] W2[l][j][k]    (axis 0, P:442 / P:215; Fig. 2(d))
+template <int P1, typename T>
+__global__ void __launch_bounds__(Cfg<P1, P1, T, 3>::NT)
+sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, const T* __restrict__ C,
+                 const T* __restrict__ U, T* __restrict__ V) {
+    using CF = Cfg<P1, P1, T, 3>;
+    using G = Geo<P1, P1, T>;
+    constexpr int E = CF::E, NT = CF::NT, R = CF::R;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T* opA = reinterpret_cast<T*>(smem_raw);
+    T* opB = opA + op_elems<P1, T>();
+    T* opC = opB + op_elems<P1, T>();
+    T* buf[2];
+    buf[0] = opC + op_elems<P1, T>();
+    buf[1] = buf[0] + CF::BUF;
+    T* W = buf[1] + CF::BUF;
+
+    load_op<P1, T, NT>(opA, A);
+    load_op<P1, T, NT>(opB, B);
+    load_op<P1, T, NT>(opC, C);
+
+    const int64_t ngroups = (N + E - 1) / E;
+    int64_t g = blockIdx.x;
+    if (g < ngroups) load_group_async<P1, P1, T, NT>(buf[0], U + g * E * G::NPTS, imin64(E, N - g * E));
+    cp_async_commit();
+    int cur = 0;
+    for (; g < ngroups; g += gridDim.x) {
+        const int64_t e0 = g * E;
+        const int ne = imin64(E, N - e0);
+        const int nlines = ne * P1 * P1;
+        cp_async_wait_all();
+        __syncthreads();
+        T* in = buf[cur];
+        const int64_t gn = g + gridDim.x;
+        if (gn < ngroups)
+            load_group_async<P1, P1, T, NT>(buf[cur ^ 1], U + gn * E * G::NPTS,
+                                            imin64(E, N - gn * E));
+        cp_async_commit();
+
+        apply_lines<P1, P1, 2, R, NT>(in, opA, nlines,
+                                      [&](int, int base, int k, T v) { W[base + k] = v; });
+        __syncthreads();
+        apply_lines<P1, P1, 1, R, NT>(W, opB, nlines,
+                                      [&](int, int base, int k, T v) { in[base + k * G::RS] = v; });
+        __syncthreads();
+        T* Vg = V + e0 * G::NPTS;
+        apply_lines<P1, P1, 0, R, NT>(in, opC, nlines, [&](int L, int, int k, T v) {
+            st_cs(Vg + Line<P1, P1, 0, T>::gofs(L, k), v);
+        });
+        cur ^= 1;
+    }
+}
+
+template <int P1, typename T>
+int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, cudaStream_t s) {
+    using CF = Cfg<P1, P1, T, 3>;
+    static int occ = 0;
+    const int64_t ngroups = (N + CF::E - 1) / CF::E;
+    const int grid = grid_for(sumfact3d_kernel<P1, T>, CF::NT, CF::SMEM, ngroups, &occ);
+    sumfact3d_kernel<P1, T><<<grid, CF::NT, CF::SMEM, s>>>(N, A, B, C, U, V);
+    return launch_status();
+}
+
+// ====================================================================== sumfact2d
+//   W[l][j] = sum_m A[j][m] U[l][m]  (axis "2" = fastest);  V[i][j] = sum_l B[i][l] W[l][j]
+template <int P1>
+__global__ void __launch_bounds__(Cfg<P1, 1, double, 3>::NT)
+sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restrict__ B,
+                 const double* __restrict__ U, double* __restrict__ V) {
+    using T = double;
+    using CF = Cfg<P1, 1, T, 3>;
+    using G = Geo<P1, 1, T>;
+    constexpr int E = CF::E, NT = CF::NT, R = CF::R;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T* opA = reinterpret_cast<T*>(smem_raw);
+    T* opB = opA + op_elems<P1, T>();
+    T* buf[2];
+    buf[0] = opB + op_elems<P1, T>();
+    buf[1] = buf[0] + CF::BUF;
+    T* W = buf[1] + CF::BUF;
+    load_op<P1, T, NT>(opA, A);
+    load_op<P1, T, NT>(opB, B);
+
+    const int64_t ngroups = (N + E - 1) / E;
+    int64_t g = blockIdx.x;
+    if (g < ngroups) load_group_async<P1, 1, T, NT>(buf[0], U + g * E * G::NPTS, imin64(E, N - g * E));
+    cp_async_commit();
+    int cur = 0;
+    for (; g < ngroups; g += gridDim.x) {
+        const int64_t e0 = g * E;
+        const int ne = imin64(E, N - e0);
+        const int nlines = ne * P1;
+        cp_async_wait_all();
+        __syncthreads();
+        T* in = buf[cur];
+        const int64_t gn = g + gridDim.x;
+        if (gn < ngroups)
+            load_group_async<P1, 1, T, NT>(buf[cur ^ 1], U + gn * E * G::NPTS, imin64(E, N - gn * E));
+        cp_async_commit();
+        apply_lines<P1, 1, 2, R, NT>(in, opA, nlines, [&](int, int base, int k, T v) { W[base + k] = v; });
+        __syncthreads();
+        T* Vg = V + e0 * G::NPTS;
+        apply_lines<P1, 1, 1, R, NT>(W, opB, nlines, [&](int L, int, int k, T v) {
+            st_cs(Vg + Line<P1, 1, 1, T>::gofs(L, k), v);
+        });
+        cur ^= 1;
+    }
+}
+
+template <int P1>
+int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* U, double* V, cudaStream_t s) {
+    using CF = Cfg<P1, 1, double, 3>;
+    static int occ = 0;
+    const int64_t ngroups = (N + CF::E - 1) / CF::E;
+    const int grid = grid_for(sumfact2d_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
+    sumfact2d_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, A, B, U, V);
+    return launch_status();
+}
+
+// ====================================================================== local_grad3
+//   ur = D along axis 2 (i), us = D along axis 1 (j), ut = D along axis 0 (k) of U[k][j][i]
+template <int P1>
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 3>::NT)
+local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ U,
+                   double* __restrict__ ur, double* __restrict__ us, double* __restrict__ ut) {
+    using T = double;
+    using CF = Cfg<P1, P1, T, 3>;
+    using G = Geo<P1, P1, T>;
+    constexpr int E = CF::E, NT = CF::NT, R = CF::R;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T* opD = reinterpret_cast<T*>(smem_raw);
+    T* buf[2];
+    buf[0] = opD + op_elems<P1, T>();
+    buf[1] = buf[0] + CF::BUF;
+    T* W = buf[1] + CF::BUF;
+    load_op<P1, T, NT>(opD, D);
+
+    const int64_t ngroups = (N + E - 1) / E;
+    int64_t g = blockIdx.x;
+    if (g < ngroups) load_group_async<P1, P1, T, NT>(buf[0], U + g * E * G::NPTS, imin64(E, N - g * E));
+    cp_async_commit();
+    int cur = 0;
+    for (; g < ngroups; g += gridDim.x) {
+        const int64_t e0 = g * E;
+        const int ne = imin64(E, N - e0);
+        const int nlines = ne * P1 * P1;
+        cp_async_wait_all();
+        __syncthreads();
+        T* in = buf[cur];
+        const int64_t gn = g + gridDim.x;
+        if (gn < ngroups)
+            load_group_async<P1, P1, T, NT>(buf[cur ^ 1], U + gn * E * G::NPTS, imin64(E, N - gn * E));
+        cp_async_commit();
+        const int64_t gbase = e0 * G::NPTS;
+        // ur -> smem (its rows are strided across threads; stored coalesced below)
+        apply_lines<P1, P1, 2, R, NT>(in, opD, nlines, [&](int, int base, int k, T v) { W[base + k] = v; });
+        apply_lines<P1, P1, 1, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
+            st_cs(us + gbase + Line<P1, P1, 1, T>::gofs(L, k), v);
+        });
+        apply_lines<P1, P1, 0, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
+            st_cs(ut + gbase + Line<P1, P1, 0, T>::gofs(L, k), v);
+        });
+        __syncthreads();
+        const int total = ne * G::NPTS;
+        for (int f = threadIdx.x; f < total; f += NT) st_cs(ur + gbase + f, W[smem_index<P1, P1, T>(f)]);
+        cur ^= 1;
+    }
+}
+
+template <int P1>
+int launch_local_grad3(int64_t N, const double* D, const double* U, double* ur, double* us, double* ut,
+                       cudaStream_t s) {
+    using CF = Cfg<P1, P1, double, 3>;
+    static int occ = 0;
+    const int64_t ngroups = (N + CF::E - 1) / CF::E;
+    const int grid = grid_for(local_grad3_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
+    local_grad3_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, D, U, ur, us, ut);
+    return launch_status();
+}
+
+// ====================================================================== local_grad3_t
+//   U = D^T along axis 2 of ur + D^T along axis 1 of us + D^T along axis 0 of ut
+//   (partial sums added in the order (r + s) + t)
+template <int P1>
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 4>::NT)
+local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ ur,
+                     const double* __restrict__ us, const double* __restrict__ ut, double* __restrict__ U) {
+    using T = double;
+    using CF = Cfg<P1, P1, T, 4>;
+    using G = Geo<P1, P1, T>;
+    constexpr int E = CF::E, NT = CF::NT, R = CF::R;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T* opT = reinterpret_cast<T*>(smem_raw);
+    T* bR = opT + op_elems<P1, T>();
+    T* bS = bR + CF::BUF;
+    T* bT = bS + CF::BUF;
+    T* W = bT + CF::BUF;
+    load_op<P1, T, NT, true>(opT, D);
+    const int64_t ngroups = (N + E - 1) / E;
+    for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
+        const int64_t e0 = g * E;
+        const int ne = imin64(E, N - e0);
+        const int nlines = ne * P1 * P1;
+        const int64_t gbase = e0 * G::NPTS;
+        __syncthreads();  // previous group fully consumed
+        load_group_async<P1, P1, T, NT>(bR, ur + gbase, ne);
+        load_group_async<P1, P1, T, NT>(bS, us + gbase, ne);
+        load_group_async<P1, P1, T, NT>(bT, ut + gbase, ne);
+        cp_async_commit();
+        cp_async_wait_all();
+        __syncthreads();
+        apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { W[base + k] = v; });
+        __syncthreads();
+        apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines,
+                                      [&](int, int base, int k, T v) { W[base + k * G::RS] += v; });
+        __syncthreads();
+        apply_lines<P1, P1, 0, R, NT>(bT, opT, nlines, [&](int L, int base, int k, T v) {
+            st_cs(U + gbase + Line<P1, P1, 0, T>::gofs(L, k), W[base + k * G::PS] + v);
+        });
+    }
+}
+
+template <int P1>
+int launch_local_grad3_t(int64_t N, const double* D, const double* ur, const double* us, const double* ut,
+                         double* U, cudaStream_t s) {
+    using CF = Cfg<P1, P1, double, 4>;
+    static int occ = 0;
+    const int64_t ngroups = (N + CF::E - 1) / CF::E;
+    const int grid = grid_for(local_grad3_t_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
+    local_grad3_t_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, D, ur, us, ut, U);
+    return launch_status();
+}
+
+// ====================================================================== ax_e
+template <int P1>
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 4>::NT)
+ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ Uin,
+            const double* __restrict__ Gm, double* __restrict__ Wout) {
+    using T = double;
+    using CF = Cfg<P1, P1, T, 4>;
+    using G = Geo<P1, P1, T>;
+    constexpr int E = CF::E, NT = CF::NT, R = CF::R;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T* opD = reinterpret_cast<T*>(smem_raw);
+    T* opT = opD + op_elems<P1, T>();
+    T* bU = opT + op_elems<P1, T>();
+    T* bR = bU + CF::BUF;
+    T* bS = bR + CF::BUF;
+    T* bT = bS + CF::BUF;
+    load_op<P1, T, NT>(opD, D);
+    load_op<P1, T, NT, true>(opT, D);
+    const int64_t ngroups = (N + E - 1) / E;
+    for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
+        const int64_t e0 = g * E;
+        const int ne = imin64(E, N - e0);
+        const int nlines = ne * P1 * P1;
+        const int64_t gbase = e0 * G::NPTS;
+        __syncthreads();
+        load_group_async<P1, P1, T, NT>(bU, Uin + gbase, ne);
+        cp_async_commit();
+        cp_async_wait_all();
+        __syncthreads();
+        apply_lines<P1, P1, 2, R, NT>(bU, opD, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
+        apply_lines<P1, P1, 1, R, NT>(bU, opD, nlines, [&](int, int base, int k, T v) { bS[base + k * G::RS] = v; });
+        apply_lines<P1, P1, 0, R, NT>(bU, opD, nlines, [&](int, int base, int k, T v) { bT[base + k * G::PS] = v; });
+        __syncthreads();
+        // geometric mixing, one thread per point: G[e][c][q]
+        const int total = ne * G::NPTS;
+        for (int f = threadIdx.x; f < total; f += NT) {
+            const int e = f / G::NPTS;
+            const int q = f - e * G::NPTS;
+            const T* gp = Gm + (e0 + e) * 6 * (int64_t)G::NPTS + q;
+            const T g0 = __ldcs(gp), g1 = __ldcs(gp + G::NPTS), g2 = __ldcs(gp + 2 * G::NPTS),
+                    g3 = __ldcs(gp + 3 * G::NPTS), g4 = __ldcs(gp + 4 * G::NPTS), g5 = __ldcs(gp + 5 * G::NPTS);
+            const int si = smem_index<P1, P1, T>(f);
+            const T r = bR[si], s = bS[si], t = bT[si];
+            bR[si] = (g0 * r + g1 * s) + g2 * t;
+            bS[si] = (g1 * r + g3 * s) + g4 * t;
+            bT[si] = (g2 * r + g4 * s) + g5 * t;
+        }
+        __syncthreads();
+        apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { bU[base + k] = v; });
+        __syncthreads();
+        apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines, [&](int, int base, int k, T v) { bU[base + k * G::RS] += v; });
+        __syncthreads();
+        apply_lines<P1, P1, 0, R, NT>(bT, opT, nlines, [&](int L, int base, int k, T v) {
+            st_cs(Wout + gbase + Line<P1, P1, 0, T>::gofs(L, k), bU[base + k * G::PS] + v);
+        });
+    }
+}
+
+template <int P1>
+int launch_ax_e(int64_t N, const double* D, const double* U, const double* Gm, double* W, cudaStream_t s) {
+    using CF = Cfg<P1, P1, double, 4>;
+    static int occ = 0;
+    const int64_t ngroups = (N + CF::E - 1) / CF::E;
+    const int grid = grid_for(ax_e_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
+    ax_e_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, D, U, Gm, W);
+    return launch_status();
+}
+
+// ---------------------------------------------------------------- P1 dispatch
+#define BC_P1_SWITCH(P1VAR, CALL)   \
+    switch (P1VAR) {                \
+        case 2: return CALL(2);     \
+        case 3: return CALL(3);     \
+        case 4: return CALL(4);     \
+        case 5: return CALL(5);     \
+        case 6: return CALL(6);     \
+        case 7: return CALL(7);     \
+        case 8: return CALL(8);     \
+        case 9: return CALL(9);     \
+        case 10: return CALL(10);   \
+        case 11: return CALL(11);   \
+        case 12: return CALL(12);   \
+        case 13: return CALL(13);   \
+        case 14: return CALL(14);   \
+        case 15: return CALL(15);   \
+        case 16: return CALL(16);   \
+        default: return BC_ERR_UNSUPPORTED; \
+    }
+
+int run_sumfact3d(int64_t N, int p, const double* A, const double* B, const double* C, const double* U,
+                  double* V, cudaStream_t s) {
+#define CALL(P) launch_sumfact3d<P, double>(N, A, B, C, U, V, s)
+    BC_P1_SWITCH(p + 1, CALL)
+#undef CALL
+}
+int run_sumfact3d_f32(int64_t N, int p, const float* A, const float* B, const float* C, const float* U,
+                      float* V, cudaStream_t s) {
+#define CALL(P) launch_sumfact3d<P, float>(N, A, B, C, U, V, s)
+    BC_P1_SWITCH(p + 1, CALL)
+#undef CALL
+}
+int run_sumfact2d(int64_t N, int p, const double* A, const double* B, const double* U, double* V,
+                  cudaStream_t s) {
+#define CALL(P) launch_sumfact2d<P>(N, A, B, U, V, s)
+    BC_P1_SWITCH(p + 1, CALL)
+#undef CALL
+}
+int run_local_grad3(int64_t N, int p, const double* D, const double* U, double* ur, double* us, double* ut,
+                    cudaStream_t s) {
+#define CALL(P) launch_local_grad3<P>(N, D, U, ur, us, ut, s)
+    BC_P1_SWITCH(p + 1, CALL)
+#undef CALL
+}
+int run_local_grad3_t(int64_t N, int p, const double* D, const double* ur, const double* us,
+                      const double* ut, double* U, cudaStream_t s) {
+#define CALL(P) launch_local_grad3_t<P>(N, D, ur, us, ut, U, s)
+    BC_P1_SWITCH(p + 1, CALL)
+#undef CALL
+}
+int run_ax_e(int64_t N, int p, const double* D, const double* U, const double* Gm, double* W, cudaStream_t s) {
+#define CALL(P) launch_ax_e<P>(N, D, U, Gm, W, s)
+    BC_P1_SWITCH(p + 1, CALL)
+#undef CALL
+}
+
+}  // namespace bc

@@ -1,0 +1,99 @@
+"""GPU parity of the CCSD(T) family (through the C ABI) against the oracle's literal
+7-deep loops.  Integer data with unequal extents (all 7 distinct) must be bitwise equal —
+a swapped extent or index cannot hide.  t3 starts non-zero (accumulate semantics)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synthetic as syn
+
+pytestmark = pytest.mark.gpu
+
+from gpu_util import assert_abs_close, to_dev, to_host  # noqa: E402
+
+
+@pytest.fixture(scope="module")
+def bc():
+    import paper_conf_icpp_nelsonrbhhjn15_b200 as m
+    return m
+
+
+def sizes(family, ext):
+    h1, h2, h3, p4, p5, p6, k = ext
+    if family == "d1":
+        return k * p4 * p5 * h1, h3 * h2 * p6 * k
+    if family == "d2":
+        return k * p4 * h1 * h2, k * h3 * p6 * p5
+    return p4 * h1, h3 * h2 * p6 * p5
+
+
+def n3(ext):
+    return int(np.prod(ext[:6]))
+
+
+EXTS = [(3, 4, 5, 6, 2, 7, 3), (9, 17, 13, 5, 3, 4, 19), (8, 8, 8, 8, 8, 8, 8), (1, 1, 1, 1, 1, 1, 1)]
+
+
+@pytest.mark.parametrize("family", ["d1", "d2", "s1"])
+@pytest.mark.parametrize("ext", EXTS)
+def test_single_variant_integer_bitwise(bc, family, ext):
+    na, nb = sizes(family, ext)
+    for v in range(1, 10):
+        t3 = syn.tensor(10, (n3(ext),), kind=syn.KIND_INT)
+        t2 = syn.tensor(20 + v, (na,), kind=syn.KIND_INT)
+        v2 = syn.tensor(40 + v, (nb,), kind=syn.KIND_INT)
+        d3 = to_dev(t3)
+        bc.ccsdt(family, v, ext, d3, to_dev(t2), to_dev(v2))
+        assert np.array_equal(to_host(d3), oracle.ccsdt(family, v, ext, t3, t2, v2)), f"{family}_{v} ext={ext}"
+
+
+@pytest.mark.parametrize("family", ["d1", "d2", "s1"])
+@pytest.mark.parametrize("ext", [(3, 4, 5, 6, 2, 7, 3), (12, 12, 12, 7, 7, 7, 21), (5, 5, 5, 3, 3, 3, 40)])
+def test_fused_integer_bitwise(bc, family, ext):
+    na, nb = sizes(family, ext)
+    t3 = syn.tensor(10, (n3(ext),), kind=syn.KIND_INT)
+    t2s = [syn.tensor(20 + v, (na,), kind=syn.KIND_INT) for v in range(1, 10)]
+    v2s = [syn.tensor(40 + v, (nb,), kind=syn.KIND_INT) for v in range(1, 10)]
+    for mask in (range(1, 10), (2, 5, 9), (7,)):
+        a = [t2s[v - 1] if v in mask else None for v in range(1, 10)]
+        d3 = to_dev(t3)
+        bc.ccsdt_fused(family, ext, d3, [None if x is None else to_dev(x) for x in a], [to_dev(x) for x in v2s])
+        assert np.array_equal(to_host(d3), oracle.ccsdt_fused(family, ext, t3, a, v2s)), f"{family} mask={list(mask)}"
+
+
+@pytest.mark.parametrize("family", ["d1", "d2"])
+@pytest.mark.parametrize("tile", [16, 24])
+def test_tile_random_tolerance(bc, family, tile):
+    """North-star tile sizes (16; BASELINE: 24), uniform data, rtol 1e-12 of S."""
+    ext = (tile,) * 7
+    na, nb = sizes(family, ext)
+    t3 = syn.tensor(10, (n3(ext),))
+    t2s = [syn.tensor(20 + v, (na,)) for v in range(1, 10)]
+    v2s = [syn.tensor(40 + v, (nb,)) for v in range(1, 10)]
+    if tile == 16:  # fused over all 9 (the oracle's 9 literal passes take too long at 24)
+        d3 = to_dev(t3)
+        bc.ccsdt_fused(family, ext, d3, [to_dev(x) for x in t2s], [to_dev(x) for x in v2s])
+        ref = oracle.ccsdt_fused(family, ext, t3, t2s, v2s)
+        S = oracle.ccsdt_abs_bound(family, ext, t3, t2s, v2s)
+        assert_abs_close(to_host(d3), ref, S, 1e-12, f"{family} fused tile {tile}")
+    v = 4
+    d3 = to_dev(t3)
+    fn = bc.lib.bc_ccsdt_d1_tile if family == "d1" else bc.lib.bc_ccsdt_d2_tile
+    import ctypes
+    st = fn(v, tile, d3.data_ptr(), to_dev(t2s[v - 1]).data_ptr(), to_dev(v2s[v - 1]).data_ptr(),
+            ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
+    assert st == 0
+    ref = oracle.ccsdt(family, v, ext, t3, t2s[v - 1], v2s[v - 1])
+    S = oracle.ccsdt_abs_bound(family, ext, t3, [t2s[v - 1] if u == v else None for u in range(1, 10)], v2s)
+    assert_abs_close(to_host(d3), ref, S, 1e-12, f"{family}_{v} tile {tile}")
+
+
+def test_energy_check(bc):
+    ext = (7, 6, 5, 4, 3, 9, 1)
+    t3 = syn.tensor(10, (n3(ext),))
+    eh = syn.tensor(60, (sum(ext[:3]),), kind=syn.KIND_RANGE, lo=-2.0, hi=-0.5)
+    ep = syn.tensor(61, (sum(ext[3:6]),), kind=syn.KIND_RANGE, lo=0.5, hi=2.0)
+    got = float(bc.check_energy(ext, to_dev(t3), to_dev(eh), to_dev(ep)).item())
+    ref = oracle.energy(ext, t3, eh, ep)
+    assert abs(got - ref) <= 1e-12 * abs(ref)
