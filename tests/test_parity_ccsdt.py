@@ -81,8 +81,8 @@ def test_tile_random_tolerance(bc, family, tile):
     d3 = to_dev(t3)
     fn = bc.lib.bc_ccsdt_d1_tile if family == "d1" else bc.lib.bc_ccsdt_d2_tile
     import ctypes
-    st = fn(v, tile, d3.data_ptr(), to_dev(t2s[v - 1]).data_ptr(), to_dev(v2s[v - 1]).data_ptr(),
-            ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
+    a, b = to_dev(t2s[v - 1]), to_dev(v2s[v - 1])  # keep both alive across the raw call
+    st = fn(v, tile, d3.data_ptr(), a.data_ptr(), b.data_ptr(), ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
     assert st == 0
     ref = oracle.ccsdt(family, v, ext, t3, t2s[v - 1], v2s[v - 1])
     S = oracle.ccsdt_abs_bound(family, ext, t3, [t2s[v - 1] if u == v else None for u in range(1, 10)], v2s)
