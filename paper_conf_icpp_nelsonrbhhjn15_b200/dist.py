@@ -1,0 +1,84 @@
+"""Multi-GPU plumbing: one process per GPU, torch.distributed for the
+process group, contiguous shard plans, and the only collectives the path has — scalar
+check reductions and the max-over-ranks of timings.  Elements and CCSD(T) tile blocks are
+independent, so no data crosses between GPUs.
+"""
+from __future__ import annotations
+
+import os
+from dataclasses import dataclass
+
+import torch
+import torch.distributed as dist
+
+
+@dataclass(frozen=True)
+class Rank:
+    rank: int
+    world: int
+    local_rank: int
+    device: torch.device
+
+
+def init(backend: str | None = None) -> Rank:
+    """Read RANK / WORLD_SIZE / LOCAL_RANK (torchrun); init the process group if world > 1.
+    backend defaults to nccl when CUDA is available, else gloo."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if torch.cuda.is_available():
+        torch.cuda.set_device(local)
+        device = torch.device("cuda", local)
+    else:
+        device = torch.device("cpu")
+    if world > 1 and not dist.is_initialized():
+        if backend is None:
+            backend = "nccl" if device.type == "cuda" else "gloo"
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group(backend=backend, rank=rank, world_size=world,
+                                device_id=device if backend == "nccl" else None)
+    return Rank(rank, world, local, device)
+
+
+def shard(n: int, rank: int, world: int) -> tuple[int, int]:
+    """Contiguous range [floor(r n / G), floor((r+1) n / G)) of n units owned by rank r."""
+    if world < 1 or not 0 <= rank < world:
+        raise ValueError("bad rank/world")
+    return (rank * n) // world, ((rank + 1) * n) // world
+
+
+def owner(unit: int, n: int, world: int) -> int:
+    """Rank owning unit `unit` under shard(); inverse of the plan."""
+    if not 0 <= unit < n:
+        raise ValueError("unit out of range")
+    r = (unit * world) // n
+    while shard(n, r, world)[1] <= unit:
+        r += 1
+    while shard(n, r, world)[0] > unit:
+        r -= 1
+    return r
+
+
+def barrier() -> None:
+    if dist.is_initialized():
+        dist.barrier()
+
+
+def all_reduce_sum_(t: torch.Tensor) -> torch.Tensor:
+    """In-place SUM of a (small) check tensor over ranks; identity when world == 1."""
+    if dist.is_initialized() and dist.get_world_size() > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return t
+
+
+def max_over_ranks(x: float, device: torch.device) -> float:
+    if dist.is_initialized() and dist.get_world_size() > 1:
+        t = torch.tensor([x], dtype=torch.float64, device=device)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+    return x
+
+
+def finalize() -> None:
+    if dist.is_initialized():
+        dist.destroy_process_group()
