@@ -8,16 +8,21 @@
 // variants (the fused form reads/writes it once for up to 9 variants).
 //
 // For one variant the unit is a small GEMM in name space:
-//   d1/s1:  X[(h3,h2), h1] = sum_k v2[h3,h2,p6,k] * t2[k,p4,p5,h1]     (M = BS^2, N = BS)
-//   d2   :  X[h3, (h1,h2)] = sum_k v2[k,h3,p6,p5] * t2[k,p4,h1,h2]     (M = BS,   N = BS^2)
-// (s1 is the K = 1 outer product t1[p4,h1] * v2[h3,h2,p6,p5]).  A cube in q-space is a
-// cube in name space for every hole permutation, so the GEMM shape is the same for all
-// variants.  Operand slices are staged in shared memory (zero-padded at block edges,
-// sign folded into the N operand), each thread accumulates a 4x4 register tile over k
-// (scalar replacement), and variants sharing a hole permutation ("class")
-// accumulate into the same registers; a class is flushed into the shared accumulator at
-// its permuted positions.  The (h1,h2,h3) <-> storage-position maps are derived here from
-// the generating rule of DESIGN.md R12 (not copied from the oracle's table).
+//   d1/s1:  X[(h3,h2), h1] = sum_k v2[h3,h2,p6,k] * t2[k,p4,p5,h1]
+//   d2   :  X[(h1,h2), h3] = sum_k t2[k,p4,h1,h2] * v2[k,h3,p6,p5]
+// (s1 is the K = 1 outer product v2[h3,h2,p6,p5] * t1[p4,h1]).  The "strided" operand
+// covers a PAIR of hole names (BS^2 values), the "broadcast" operand the third (BS).  A
+// cube in q-space is a cube in name space for every hole permutation, so the GEMM shape
+// is the same for all variants.  Operand slices for (variant, k-chunk) stages are staged
+// in shared memory by cp.async (zero-filled at block edges) one stage ahead of the
+// compute.  Each thread accumulates a TS x TB register tile over k (scalar replacement,
+// P:553-558): TS strided values at lane stride (conflict-free scalar reads) times TB
+// broadcast values (16-byte reads); the variant's sign flips the broadcast values' sign
+// bit.  Variants sharing a hole permutation ("class") accumulate into the same
+// registers; a class is flushed into the shared accumulator cube at its permuted
+// positions.  The cube has odd strides (1, BS+1, (BS+1)^2) on every axis, so the flush is
+// bank-conflict free for any permutation.  The (h1,h2,h3) <-> storage-position maps are
+// derived here from the generating rule of DESIGN.md R12 (not copied from the oracle).
 #include "common.cuh"
 
 namespace bc {
@@ -83,178 +88,204 @@ struct CcsdtParams {
     int ncube[3];     // cubes along q1, q2, q3
 };
 
+// Per cube side BS: register tile TS (strided operand, one value per lane-stride) x TB
+// (broadcast operand, 16-byte smem reads), k chunk KC.
 template <int BS>
-struct CcTile {
-    static constexpr int TILES = BS * BS * BS / 16;          // 4x4 register tiles
+struct CcTile;
+template <>
+struct CcTile<16> { static constexpr int TS = 4, TB = 8; };
+template <>
+struct CcTile<12> { static constexpr int TS = 4, TB = 4; };
+template <>
+struct CcTile<8> { static constexpr int TS = 2, TB = 4; };
+
+template <int BS>
+struct CcGeo {
+    static constexpr int TS = CcTile<BS>::TS, TB = CcTile<BS>::TB;
+    static constexpr int SD = BS * BS;            // strided dim: a PAIR of hole names
+    static constexpr int BD = BS;                 // broadcast dim: the third hole name
+    static constexpr int MS = SD / TS;            // lanes along the strided dim
+    static constexpr int NB = BD / TB;
+    static constexpr int TILES = MS * NB;
     static constexpr int NT = (TILES + 31) / 32 * 32;
-    static constexpr int KC = 16;                            // k chunk
-    static constexpr int MN2 = BS * BS + 2;                  // padded smem row (x doubles)
-    static constexpr int MN1 = BS + 2;
-    static constexpr size_t SMEM = (size_t)(BS * BS * BS + KC * MN2 + KC * MN2) * sizeof(double);
+    static constexpr int KC = (BS >= 16) ? 8 : 16;  // k chunk per pipeline stage
+    static constexpr int SS = SD + 1;             // odd row stride: conflict-free both ways
+    static constexpr int SB = BD + 2;             // even row stride: 16-byte rows
+    static constexpr int CST = BS + 1;            // accumulator cube strides 1, CST, CST^2 (all odd)
+    static constexpr int ACC = BS * CST * CST;
+    static constexpr int STAGE = KC * SS + KC * SB;  // even (KC even): stage bases stay 16-byte aligned
+    static constexpr size_t SMEM = (size_t)(ACC + (ACC & 1) + 2 * STAGE + 2) * sizeof(double);
 };
 
-template <int FAM, int BS>
-__global__ void __launch_bounds__(CcTile<BS>::NT) ccsdt_kernel(const CcsdtParams P) {
-    using TT = CcTile<BS>;
-    constexpr int NT = TT::NT, KC = TT::KC;
-    constexpr int M = (FAM == FAM_D2) ? BS : BS * BS;   // v2 side
-    constexpr int N = (FAM == FAM_D2) ? BS * BS : BS;   // t2 / t1 side
-    constexpr int SA = M + 2, SB = N + 2;                // smem row strides (16B-aligned rows)
-    constexpr int MT = M / 4;
-    extern __shared__ __align__(16) double sm[];
-    double* acc_s = sm;                  // BS^3 accumulator, index q0 + BS*(q1 + BS*q2)
-    double* As = acc_s + BS * BS * BS;   // [KC][SA]
-    double* Bs = As + KC * SA;           // [KC][SB]
+__device__ __forceinline__ void cp_async_8_zfill(void* dst, const void* src, bool valid) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(smem_u32(dst)), "l"(src),
+                 "r"(valid ? 8 : 0));
+}
 
-    // ---- unit decode
+__device__ __forceinline__ double flip_sign(double x, uint32_t mask_hi) {
+    return __hiloint2double(__double2hiint(x) ^ (int)mask_hi, __double2loint(x));
+}
+
+template <int FAM, int BS>
+__global__ void __launch_bounds__(CcGeo<BS>::NT) ccsdt_kernel(const CcsdtParams P) {
+    using CG = CcGeo<BS>;
+    constexpr int NT = CG::NT, KC = CG::KC, TS = CG::TS, TB = CG::TB, MS = CG::MS;
+    constexpr int SD = CG::SD, BD = CG::BD, SS = CG::SS, SB = CG::SB, CST = CG::CST;
+    extern __shared__ __align__(16) double sm[];
+    double* acc_s = sm;
+    double* stage0 = sm + ((CG::ACC + 1) & ~1);
+
+    // ---- unit decode: cube (o, len) in the hole positions, plane qv in the particle ones
     const int ncubes = P.ncube[0] * P.ncube[1] * P.ncube[2];
     const int cube = blockIdx.x % ncubes;
     const int plane = blockIdx.x / ncubes;
     int o[3], len[3];
-    {
-        const int c0 = cube % P.ncube[0];
-        const int c1 = (cube / P.ncube[0]) % P.ncube[1];
-        const int c2 = cube / (P.ncube[0] * P.ncube[1]);
-        o[0] = c0 * BS;
-        o[1] = c1 * BS;
-        o[2] = c2 * BS;
-        for (int q = 0; q < 3; ++q) len[q] = min(BS, P.qe[q] - o[q]);
-    }
+    o[0] = (cube % P.ncube[0]) * BS;
+    o[1] = ((cube / P.ncube[0]) % P.ncube[1]) * BS;
+    o[2] = (cube / (P.ncube[0] * P.ncube[1])) * BS;
+    for (int q = 0; q < 3; ++q) len[q] = min(BS, P.qe[q] - o[q]);
     int qv[3];
     qv[0] = plane % P.qe[3];
     qv[1] = (plane / P.qe[3]) % P.qe[4];
     qv[2] = plane / (P.qe[3] * P.qe[4]);
 
-    for (int i = threadIdx.x; i < BS * BS * BS; i += NT) acc_s[i] = 0.0;
+    for (int i = threadIdx.x; i < CG::ACC; i += NT) acc_s[i] = 0.0;
 
     const int H1 = P.ext[N_H1], H2 = P.ext[N_H2], H3 = P.ext[N_H3];
     const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6];
     const int K = (FAM == FAM_S1) ? 1 : P.ext[N_K];
+    const int nchunk = (K + KC - 1) / KC;
+    const int nstage = P.nentry * nchunk;
 
-    const int tt = threadIdx.x;
-    const bool has_tile = tt < TT::TILES;
-    const int mt = tt % MT, nt = tt / MT;
-
-    int entry = 0;
-    for (int c = 0; c < P.ncls; ++c) {
-        // name-space origin / length of the cube for this class's hole permutation
+    // stage (entry e, chunk c) -> smem buffer b: strided operand Ss[kk][sd], broadcast Bb[kk][bd]
+    auto issue = [&](int st, int b) {
+        const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+        const int kc = min(KC, K - k0);
+        double* Ss = stage0 + b * CG::STAGE;
+        double* Bb = Ss + KC * SS;
+        const int c = P.ecls[e];
         const int hp1 = P.hpos[c][0], hp2 = P.hpos[c][1], hp3 = P.hpos[c][2];
         const int O1 = o[hp1], O2 = o[hp2], O3 = o[hp3];
         const int L1 = len[hp1], L2 = len[hp2], L3 = len[hp3];
-        double acc[4][4];
-#pragma unroll
-        for (int a = 0; a < 4; ++a)
-#pragma unroll
-            for (int b = 0; b < 4; ++b) acc[a][b] = 0.0;
-
-        for (; entry < P.nentry && P.ecls[entry] == c; ++entry) {
-            const double* __restrict__ tA = P.opA[entry];
-            const double* __restrict__ vB = P.opB[entry];
-            const double sg = P.sign[entry];
-            const int p4 = qv[P.ppos[entry][0] - 3];
-            const int p5 = qv[P.ppos[entry][1] - 3];
-            const int p6 = qv[P.ppos[entry][2] - 3];
-            for (int k0 = 0; k0 < K; k0 += KC) {
-                const int kc = min(KC, K - k0);
-                __syncthreads();
-                // ---- stage the v2 slice (M side) and the t2/t1 slice (N side, signed)
-                if constexpr (FAM == FAM_D1 || FAM == FAM_S1) {
-                    // As[kk][i3 + BS*i2] = v2[h3, h2, p6, k]   (d1)  |  v2[h3, h2, p6, p5] (s1)
-                    for (int x = threadIdx.x; x < KC * M; x += NT) {
-                        const int kk = x / M, m = x - kk * M;
-                        const int i2 = m / BS, i3 = m - i2 * BS;
-                        double v = 0.0;
-                        if (kk < kc && i3 < L3 && i2 < L2) {
-                            const int last = (FAM == FAM_S1) ? p5 : (k0 + kk);
-                            v = __ldg(vB + (O3 + i3) + (int64_t)H3 * ((O2 + i2) + (int64_t)H2 * (p6 + (int64_t)P6 * last)));
-                        }
-                        As[kk * SA + m] = v;
-                    }
-                    // Bs[kk][i1] = s * t2[k, p4, p5, h1]  (d1)  |  s * t1[p4, h1] (s1)
-                    for (int x = threadIdx.x; x < KC * N; x += NT) {
-                        const int i1 = x / KC, kk = x - i1 * KC;
-                        double v = 0.0;
-                        if (kk < kc && i1 < L1) {
-                            if constexpr (FAM == FAM_S1)
-                                v = sg * __ldg(tA + p4 + (int64_t)P4 * (O1 + i1));
-                            else
-                                v = sg * __ldg(tA + (k0 + kk) + (int64_t)K * (p4 + (int64_t)P4 * (p5 + (int64_t)P5 * (O1 + i1))));
-                        }
-                        Bs[kk * SB + i1] = v;
-                    }
-                } else {
-                    // As[kk][i3] = v2[k, h3, p6, p5]
-                    for (int x = threadIdx.x; x < KC * M; x += NT) {
-                        const int i3 = x / KC, kk = x - i3 * KC;
-                        double v = 0.0;
-                        if (kk < kc && i3 < L3)
-                            v = __ldg(vB + (k0 + kk) + (int64_t)K * ((O3 + i3) + (int64_t)H3 * (p6 + (int64_t)P6 * p5)));
-                        As[kk * SA + i3] = v;
-                    }
-                    // Bs[kk][i1 + BS*i2] = s * t2[k, p4, h1, h2]
-                    for (int x = threadIdx.x; x < KC * N; x += NT) {
-                        const int n = x / KC, kk = x - n * KC;
-                        const int i2 = n / BS, i1 = n - i2 * BS;
-                        double v = 0.0;
-                        if (kk < kc && i1 < L1 && i2 < L2)
-                            v = sg * __ldg(tA + (k0 + kk) + (int64_t)K * (p4 + (int64_t)P4 * ((O1 + i1) + (int64_t)H1 * (O2 + i2))));
-                        Bs[kk * SB + n] = v;
-                    }
+        const int p4 = qv[P.ppos[e][0] - 3], p5 = qv[P.ppos[e][1] - 3], p6 = qv[P.ppos[e][2] - 3];
+        const double* __restrict__ tA = P.opA[e];
+        const double* __restrict__ vB = P.opB[e];
+        if constexpr (FAM == FAM_D1 || FAM == FAM_S1) {
+            // Ss[kk][i3 + BS*i2] = v2[h3,h2,p6,k] (d1) | v2[h3,h2,p6,p5] (s1): contiguous along h3
+            for (int x = threadIdx.x; x < KC * SD; x += NT) {
+                const int kk = x / SD, sd = x - kk * SD;
+                const int i2 = sd / BS, i3 = sd - i2 * BS;
+                const bool ok = kk < kc && i3 < L3 && i2 < L2;
+                const int last = (FAM == FAM_S1) ? p5 : (k0 + kk);
+                const double* src = vB + (ok ? (O3 + i3) + (int64_t)H3 * ((O2 + i2) + (int64_t)H2 * (p6 + (int64_t)P6 * last)) : 0);
+                cp_async_8_zfill(Ss + kk * SS + sd, src, ok);
+            }
+            // Bb[kk][i1] = t2[k,p4,p5,h1] (d1) | t1[p4,h1] (s1): contiguous along k
+            for (int x = threadIdx.x; x < KC * BD; x += NT) {
+                const int i1 = x / KC, kk = x - i1 * KC;
+                const bool ok = kk < kc && i1 < L1;
+                int64_t off = 0;
+                if (ok) {
+                    if constexpr (FAM == FAM_S1)
+                        off = p4 + (int64_t)P4 * (O1 + i1);
+                    else
+                        off = (k0 + kk) + (int64_t)K * (p4 + (int64_t)P4 * (p5 + (int64_t)P5 * (O1 + i1)));
                 }
-                __syncthreads();
-                if (has_tile) {
-                    for (int kk = 0; kk < kc; ++kk) {
-                        const double2 a01 = *reinterpret_cast<const double2*>(As + kk * SA + 4 * mt);
-                        const double2 a23 = *reinterpret_cast<const double2*>(As + kk * SA + 4 * mt + 2);
-                        const double2 b01 = *reinterpret_cast<const double2*>(Bs + kk * SB + 4 * nt);
-                        const double2 b23 = *reinterpret_cast<const double2*>(Bs + kk * SB + 4 * nt + 2);
-                        const double av[4] = {a01.x, a01.y, a23.x, a23.y};
-                        const double bv[4] = {b01.x, b01.y, b23.x, b23.y};
+                cp_async_8_zfill(Bb + kk * SB + i1, tA + off, ok);
+            }
+        } else {
+            // Ss[kk][i1 + BS*i2] = t2[k,p4,h1,h2]: contiguous along k
+            for (int x = threadIdx.x; x < KC * SD; x += NT) {
+                const int sd = x / KC, kk = x - sd * KC;
+                const int i2 = sd / BS, i1 = sd - i2 * BS;
+                const bool ok = kk < kc && i1 < L1 && i2 < L2;
+                const double* src = tA + (ok ? (k0 + kk) + (int64_t)K * (p4 + (int64_t)P4 * ((O1 + i1) + (int64_t)H1 * (O2 + i2))) : 0);
+                cp_async_8_zfill(Ss + kk * SS + sd, src, ok);
+            }
+            // Bb[kk][i3] = v2[k,h3,p6,p5]: contiguous along k
+            for (int x = threadIdx.x; x < KC * BD; x += NT) {
+                const int i3 = x / KC, kk = x - i3 * KC;
+                const bool ok = kk < kc && i3 < L3;
+                const double* src = vB + (ok ? (k0 + kk) + (int64_t)K * ((O3 + i3) + (int64_t)H3 * (p6 + (int64_t)P6 * p5)) : 0);
+                cp_async_8_zfill(Bb + kk * SB + i3, src, ok);
+            }
+        }
+    };
+
+    const int tid = threadIdx.x;
+    const bool has_tile = tid < CG::TILES;
+    const int ms = tid % MS, nb = tid / MS;
+
+    double acc[TS][TB];
 #pragma unroll
-                        for (int a = 0; a < 4; ++a)
+    for (int a = 0; a < TS; ++a)
 #pragma unroll
-                            for (int b = 0; b < 4; ++b) acc[a][b] = fma(av[a], bv[b], acc[a][b]);
+        for (int b = 0; b < TB; ++b) acc[a][b] = 0.0;
+
+    if (nstage > 0) issue(0, 0);
+    cp_async_commit();
+    for (int st = 0; st < nstage; ++st) {
+        cp_async_wait_all();
+        __syncthreads();
+        if (st + 1 < nstage) issue(st + 1, (st + 1) & 1);
+        cp_async_commit();
+        const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+        const int kc = min(KC, K - k0);
+        const double* Ss = stage0 + (st & 1) * CG::STAGE;
+        const double* Bb = Ss + KC * SS;
+        const uint32_t smask = P.sign[e] < 0 ? 0x80000000u : 0u;
+        if (has_tile) {
+#pragma unroll 4
+            for (int kk = 0; kk < kc; ++kk) {
+                double sv[TS], bv[TB];
+#pragma unroll
+                for (int a = 0; a < TS; ++a) sv[a] = Ss[kk * SS + ms + MS * a];
+#pragma unroll
+                for (int b = 0; b < TB; b += 2) {
+                    const double2 t = *reinterpret_cast<const double2*>(Bb + kk * SB + TB * nb + b);
+                    bv[b] = flip_sign(t.x, smask);
+                    bv[b + 1] = flip_sign(t.y, smask);
+                }
+#pragma unroll
+                for (int a = 0; a < TS; ++a)
+#pragma unroll
+                    for (int b = 0; b < TB; ++b) acc[a][b] = fma(sv[a], bv[b], acc[a][b]);
+            }
+        }
+        // last chunk of the last entry of a class: flush the class into the cube
+        const bool last_chunk = (k0 + KC >= K);
+        const bool class_end = last_chunk && (e + 1 == P.nentry || P.ecls[e + 1] != P.ecls[e]);
+        if (class_end) {
+            if (has_tile) {
+                const int c = P.ecls[e];
+                const int strq[3] = {1, CST, CST * CST};
+                const int s1 = strq[P.hpos[c][0]], s2 = strq[P.hpos[c][1]], s3 = strq[P.hpos[c][2]];
+#pragma unroll
+                for (int a = 0; a < TS; ++a) {
+                    const int sd = ms + MS * a;
+                    const int hi = sd / BS, lo = sd - hi * BS;
+                    // d1/s1: strided = (i3 = lo, i2 = hi), broadcast = i1;  d2: strided = (i1 = lo, i2 = hi), broadcast = i3
+                    const int base = (FAM == FAM_D2) ? (lo * s1 + hi * s2) : (lo * s3 + hi * s2);
+                    const int sb = (FAM == FAM_D2) ? s3 : s1;
+#pragma unroll
+                    for (int b = 0; b < TB; ++b) {
+                        acc_s[base + (TB * nb + b) * sb] += acc[a][b];
+                        acc[a][b] = 0.0;
                     }
                 }
             }
         }
-        // ---- flush this class into the cube accumulator at its permuted positions
-        if (has_tile) {
-#pragma unroll
-            for (int a = 0; a < 4; ++a)
-#pragma unroll
-                for (int b = 0; b < 4; ++b) {
-                    const int m = 4 * mt + a, n = 4 * nt + b;
-                    int i1, i2, i3;
-                    if constexpr (FAM == FAM_D2) {
-                        i3 = m;
-                        i2 = n / BS;
-                        i1 = n - i2 * BS;
-                    } else {
-                        i2 = m / BS;
-                        i3 = m - i2 * BS;
-                        i1 = n;
-                    }
-                    if (i1 < L1 && i2 < L2 && i3 < L3) {
-                        int ql[3];
-                        ql[hp1] = i1;
-                        ql[hp2] = i2;
-                        ql[hp3] = i3;
-                        acc_s[ql[0] + BS * (ql[1] + BS * ql[2])] += acc[a][b];
-                    }
-                }
-        }
     }
     __syncthreads();
-    // ---- t3 += accumulator (read and written once)
+    // ---- t3 += accumulator (read and written once, coalesced along q1)
     const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
                           (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
-    for (int i = threadIdx.x; i < BS * BS * BS; i += NT) {
-        const int q0 = i % BS, q1 = (i / BS) % BS, q2 = i / (BS * BS);
-        if (q0 < len[0] && q1 < len[1] && q2 < len[2]) {
-            double* p = P.t3 + pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2));
-            *p += acc_s[i];
-        }
+    const int nvol = len[0] * len[1] * len[2];
+    for (int i = tid; i < nvol; i += NT) {
+        const int q0 = i % len[0], r = i / len[0];
+        const int q1 = r % len[1], q2 = r / len[1];
+        double* p = P.t3 + pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2));
+        *p += acc_s[q0 + CST * (q1 + CST * q2)];
     }
 }
 
@@ -276,7 +307,7 @@ static int choose_bs(const int* qe) {
 
 template <int FAM, int BS>
 static int launch_ccsdt_bs(const CcsdtParams& P, cudaStream_t s) {
-    using TT = CcTile<BS>;
+    using TT = CcGeo<BS>;
     static bool init = false;
     if (!init) {
         cudaFuncSetAttribute(ccsdt_kernel<FAM, BS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TT::SMEM);

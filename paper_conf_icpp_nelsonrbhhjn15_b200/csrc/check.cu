@@ -41,30 +41,48 @@ struct EnergyDims {
     int h1, h2, h3, p4, p5, p6;
 };
 
-// canonical t3 order (h3,h2,h1,p6,p5,p4), Fortran (h3 fastest)
+// canonical t3 order (h3,h2,h1,p6,p5,p4), Fortran (h3 fastest) = [particle plane][hole index]
+// Blocks stride over particle planes; the hole part of the denominator, (e3+e2)+e1, is
+// tabulated once per block in shared memory (when it fits), so the per-element work is
+// ((dh - f6) - f5) - f4: the oracle's summation order.
+constexpr int EN_TAB = 4096;
 __global__ void __launch_bounds__(RED_NT) energy_partial(EnergyDims d, const double* __restrict__ t3,
                                                         const double* __restrict__ eh, const double* __restrict__ ep,
                                                         double* __restrict__ part) {
     __shared__ double sh[RED_NT / 32];
-    const int64_t n = (int64_t)d.h1 * d.h2 * d.h3 * d.p4 * d.p5 * d.p6;
+    __shared__ double dh[EN_TAB];
+    const int nh = d.h1 * d.h2 * d.h3;
+    const int np = d.p4 * d.p5 * d.p6;
     const double* e1 = eh;
     const double* e2 = eh + d.h1;
     const double* e3 = eh + d.h1 + d.h2;
     const double* f4 = ep;
     const double* f5 = ep + d.p4;
     const double* f6 = ep + d.p4 + d.p5;
+    const bool tab = nh <= EN_TAB;
+    if (tab)
+        for (int i = threadIdx.x; i < nh; i += RED_NT) {
+            const int h3 = i % d.h3, h2 = (i / d.h3) % d.h2, h1 = i / (d.h3 * d.h2);
+            dh[i] = (e3[h3] + e2[h2]) + e1[h1];
+        }
+    __syncthreads();
     double s = 0.0;
-    for (int64_t i = blockIdx.x * (int64_t)RED_NT + threadIdx.x; i < n; i += (int64_t)gridDim.x * RED_NT) {
-        int64_t r = i;
-        const int h3 = (int)(r % d.h3); r /= d.h3;
-        const int h2 = (int)(r % d.h2); r /= d.h2;
-        const int h1 = (int)(r % d.h1); r /= d.h1;
-        const int p6 = (int)(r % d.p6); r /= d.p6;
-        const int p5 = (int)(r % d.p5); r /= d.p5;
-        const int p4 = (int)r;
-        const double den = ((((e3[h3] + e2[h2]) + e1[h1]) - f6[p6]) - f5[p5]) - f4[p4];
-        const double t = __ldcs(t3 + i);
-        s += t * t / den;
+    for (int pl = blockIdx.x; pl < np; pl += gridDim.x) {
+        const int p6 = pl % d.p6, p5 = (pl / d.p6) % d.p5, p4 = pl / (d.p6 * d.p5);
+        const double a6 = f6[p6], a5 = f5[p5], a4 = f4[p4];
+        const double* row = t3 + (int64_t)pl * nh;
+        for (int i = threadIdx.x; i < nh; i += RED_NT) {
+            double h;
+            if (tab) {
+                h = dh[i];
+            } else {
+                const int h3 = i % d.h3, h2 = (i / d.h3) % d.h2, h1 = i / (d.h3 * d.h2);
+                h = (e3[h3] + e2[h2]) + e1[h1];
+            }
+            const double den = ((h - a6) - a5) - a4;
+            const double t = __ldcs(row + i);
+            s += t * t / den;
+        }
     }
     s = block_sum(s, sh);
     if (threadIdx.x == 0) part[blockIdx.x] = s;
@@ -89,8 +107,9 @@ int run_sumsq(int64_t n, const double* x, double* ws, cudaStream_t s) {
 
 int run_energy(const int* ext7, const double* t3, const double* eh, const double* ep, double* ws, cudaStream_t s) {
     EnergyDims d{ext7[0], ext7[1], ext7[2], ext7[3], ext7[4], ext7[5]};
-    const int64_t n = (int64_t)d.h1 * d.h2 * d.h3 * d.p4 * d.p5 * d.p6;
-    const int nb = red_blocks(n);
+    const int np = d.p4 * d.p5 * d.p6;
+    int nb = red_blocks((int64_t)np * RED_NT * 8);
+    if (nb > np) nb = np;
     energy_partial<<<nb, RED_NT, 0, s>>>(d, t3, eh, ep, ws + 8);
     int st = launch_status();
     if (st) return st;

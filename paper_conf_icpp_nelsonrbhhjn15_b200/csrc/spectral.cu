@@ -117,67 +117,69 @@ struct Line {
 };
 
 // out(L, base, k, value): consumer of one output value.
-// Applies op (P1 x P1 in smem, row stride OS) along AXIS of the lines [0, nlines):
-//     y(L, k) = sum_{n=0..P1-1} op[k][n] * x(L, n)       (ascending n)
+// Applies an operator along AXIS of the lines [0, nlines):
+//     y(L, k) = sum_{n=0..P1-1} M[k][n] * x(L, n)       (ascending n)
+// with opT[n][k] = M[k][n] staged in smem (row stride OS).  Outer-product form: the
+// thread streams x(L, n) for its R lines and updates all P1*R accumulators, so each
+// 16-byte broadcast operator load feeds 2R FMAs and there are P1*R independent FMA
+// chains per thread.  All reads of a line precede the writes of that line and every
+// line is read by exactly one thread, so `out` may overwrite the line in place.
 template <int P1, int NA, int AXIS, int R, int NT, typename T, typename Out>
-__device__ __forceinline__ void apply_lines(const T* __restrict__ in, const T* __restrict__ op,
-                                            int nlines, Out out) {
+__device__ __forceinline__ void apply_lines(const T* in, const T* __restrict__ opT, int nlines, Out out) {
     using G = Geo<P1, NA, T>;
     using LN = Line<P1, NA, AXIS, T>;
     using P2 = typename Pair<T>::type;
+    constexpr int KP = P1 / 2;
     for (int L0 = threadIdx.x; L0 < nlines; L0 += R * NT) {
-        T x[R][P1];
         int base[R];
 #pragma unroll
         for (int r = 0; r < R; ++r) {
             int L = L0 + r * NT;
             L = (L < nlines) ? L : L0;
             base[r] = LN::base(L);
-            if constexpr (AXIS == 2 && G::VEC_ROWS) {
-#pragma unroll
-                for (int n = 0; n < P1; n += 2) {
-                    const P2 v = *reinterpret_cast<const P2*>(in + base[r] + n);
-                    x[r][n] = v.x;
-                    x[r][n + 1] = v.y;
-                }
-            } else {
-#pragma unroll
-                for (int n = 0; n < P1; ++n) x[r][n] = in[base[r] + n * LN::STRIDE];
-            }
         }
+        T acc[P1][R];
+#pragma unroll
+        for (int k = 0; k < P1; ++k)
+#pragma unroll
+            for (int r = 0; r < R; ++r) acc[k][r] = T(0);
 #pragma unroll 1
-        for (int k = 0; k < P1; ++k) {  // not unrolled: keeps only the lines in registers
-            T acc[R];
+        for (int n = 0; n < P1; ++n) {
+            T x[R];
 #pragma unroll
-            for (int r = 0; r < R; ++r) acc[r] = T(0);
+            for (int r = 0; r < R; ++r) x[r] = in[base[r] + n * LN::STRIDE];
+            const T* orow = opT + n * G::OS;
 #pragma unroll
-            for (int n = 0; n + 1 < P1; n += 2) {
-                const P2 o = *reinterpret_cast<const P2*>(op + k * G::OS + n);
+            for (int k2 = 0; k2 < KP; ++k2) {
+                const P2 o = reinterpret_cast<const P2*>(orow)[k2];
 #pragma unroll
                 for (int r = 0; r < R; ++r) {
-                    acc[r] = fma(o.x, x[r][n], acc[r]);
-                    acc[r] = fma(o.y, x[r][n + 1], acc[r]);
+                    acc[2 * k2][r] = fma(o.x, x[r], acc[2 * k2][r]);
+                    acc[2 * k2 + 1][r] = fma(o.y, x[r], acc[2 * k2 + 1][r]);
                 }
             }
             if constexpr (P1 & 1) {
-                const T o = op[k * G::OS + P1 - 1];
+                const T o = orow[P1 - 1];
 #pragma unroll
-                for (int r = 0; r < R; ++r) acc[r] = fma(o, x[r][P1 - 1], acc[r]);
+                for (int r = 0; r < R; ++r) acc[P1 - 1][r] = fma(o, x[r], acc[P1 - 1][r]);
             }
-#pragma unroll
-            for (int r = 0; r < R; ++r)
-                if (L0 + r * NT < nlines) out(L0 + r * NT, base[r], k, acc[r]);
         }
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+            if (L0 + r * NT < nlines) {
+#pragma unroll
+                for (int k = 0; k < P1; ++k) out(L0 + r * NT, base[r], k, acc[k][r]);
+            }
     }
 }
 
-// operator staging: op_s[k][n] = M[k][n] (TRANSPOSE = false) or M[n][k] (true)
+// operator staging: opT[n][k] = M[k][n], M = Mat (TRANSPOSE = false) or Mat^T (true)
 template <int P1, typename T, int NT, bool TRANSPOSE = false>
-__device__ __forceinline__ void load_op(T* __restrict__ op_s, const T* __restrict__ M) {
+__device__ __forceinline__ void load_op(T* __restrict__ op_s, const T* __restrict__ Mat) {
     constexpr int OS = (P1 + 1) & ~1;
     for (int i = threadIdx.x; i < P1 * OS; i += NT) {
-        const int k = i / OS, n = i - (i / OS) * OS;
-        op_s[i] = (n < P1) ? (TRANSPOSE ? M[n * P1 + k] : M[k * P1 + n]) : T(0);
+        const int n = i / OS, k = i - (i / OS) * OS;
+        op_s[i] = (k < P1) ? (TRANSPOSE ? Mat[n * P1 + k] : Mat[k * P1 + n]) : T(0);
     }
 }
 
@@ -190,19 +192,22 @@ __host__ __device__ __forceinline__ int imin64(int64_t a, int64_t b) { return (i
 
 // ---------------------------------------------------------------- launch configuration
 // The fixed variant table (north star: "settled by ncu measurement and recorded in a
-// small fixed table"): elements per CTA E, threads NT, lines per thread R.
+// small fixed table"): elements per CTA group E, threads NT, lines per thread R, number
+// of element buffers NBUF.  All stages run in place, so a kernel needs one buffer per
+// live field (+1 for the prefetch of the next group).
 template <int P1, int NA, typename T, int NBUF>
 struct Cfg {
     using G = Geo<P1, NA, T>;
-    static constexpr int BUF_BYTES = 36 * 1024;  // per element-group buffer
+    static constexpr int BUF_BYTES = 36 * 1024;  // target bytes per element-group buffer
     static constexpr int E0 = BUF_BYTES / (G::ES * (int)sizeof(T));
     static constexpr int E = E0 < 2 ? 1 : (E0 & ~1);  // even: groups of odd-P1 elements stay 16B-aligned
     static constexpr int R = 2;
     static constexpr int LINES = E * NA * P1;  // lines per axis per group (E * NPTS / P1)
     static constexpr int NT0 = ((LINES + R - 1) / R + 31) / 32 * 32;
     static constexpr int NT = NT0 < 64 ? 64 : (NT0 > 512 ? 512 : NT0);
-    static constexpr int BUF = (E * G::ES + (16 / (int)sizeof(T)) - 1) / (16 / (int)sizeof(T)) * (16 / (int)sizeof(T));
-    static constexpr size_t SMEM = (size_t)NBUF * BUF * sizeof(T) + 4 * op_elems<P1, T>() * sizeof(T);
+    static constexpr int VEC = 16 / (int)sizeof(T);
+    static constexpr int BUF = (E * G::ES + VEC - 1) / VEC * VEC;
+    static constexpr size_t SMEM = (size_t)NBUF * BUF * sizeof(T) + 2 * op_elems<P1, T>() * sizeof(T);
 };
 
 template <typename KernelT>
@@ -217,121 +222,105 @@ int grid_for(KernelT kernel, int nt, size_t smem, int64_t ngroups, int* occ_cach
     return imin64(ngroups, cap);
 }
 
-// ====================================================================== sumfact3d
-//   S1 W1[l][m][k] = sum_n A[k][n] U[l][m][n]     (axis 2, P:440 / Fig. 2(b) P:213)
-//   S2 W2[l][j][k] = sum_m B[j][m] W1[l][m][k]    (axis 1, P:441 / P:214)
-//   S3 V [i][j][k] = sum_l C[i][l] W2[l][j][k]    (axis 0, P:442 / P:215; Fig. 2(d))
-template <int P1, typename T>
-__global__ void __launch_bounds__(Cfg<P1, P1, T, 3>::NT)
-sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, const T* __restrict__ C,
-                 const T* __restrict__ U, T* __restrict__ V) {
-    using CF = Cfg<P1, P1, T, 3>;
-    using G = Geo<P1, P1, T>;
-    constexpr int E = CF::E, NT = CF::NT, R = CF::R;
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    T* opA = reinterpret_cast<T*>(smem_raw);
-    T* opB = opA + op_elems<P1, T>();
-    T* opC = opB + op_elems<P1, T>();
-    T* buf[2];
-    buf[0] = opC + op_elems<P1, T>();
-    buf[1] = buf[0] + CF::BUF;
-    T* W = buf[1] + CF::BUF;
-
-    load_op<P1, T, NT>(opA, A);
-    load_op<P1, T, NT>(opB, B);
-    load_op<P1, T, NT>(opC, C);
-
+// Group loop with a one-group-ahead cp.async prefetch of the single input field:
+//   body(in, e0, ne) processes group starting at element e0 held in smem `in`.
+template <int P1, int NA, typename T, int NT, int E, int BUF, typename Body>
+__device__ __forceinline__ void group_loop_prefetch(int64_t N, const T* __restrict__ src, T* buf0, Body body) {
+    using G = Geo<P1, NA, T>;
     const int64_t ngroups = (N + E - 1) / E;
     int64_t g = blockIdx.x;
-    if (g < ngroups) load_group_async<P1, P1, T, NT>(buf[0], U + g * E * G::NPTS, imin64(E, N - g * E));
+    if (g < ngroups) load_group_async<P1, NA, T, NT>(buf0, src + g * E * G::NPTS, imin64(E, N - g * E));
     cp_async_commit();
     int cur = 0;
     for (; g < ngroups; g += gridDim.x) {
         const int64_t e0 = g * E;
-        const int ne = imin64(E, N - e0);
-        const int nlines = ne * P1 * P1;
         cp_async_wait_all();
-        __syncthreads();
-        T* in = buf[cur];
+        __syncthreads();  // group g landed; everyone is done with the other buffer
+        T* in = buf0 + cur * BUF;
         const int64_t gn = g + gridDim.x;
         if (gn < ngroups)
-            load_group_async<P1, P1, T, NT>(buf[cur ^ 1], U + gn * E * G::NPTS,
-                                            imin64(E, N - gn * E));
+            load_group_async<P1, NA, T, NT>(buf0 + (cur ^ 1) * BUF, src + gn * E * G::NPTS, imin64(E, N - gn * E));
         cp_async_commit();
+        body(in, e0, imin64(E, N - e0));
+        cur ^= 1;
+    }
+}
 
-        apply_lines<P1, P1, 2, R, NT>(in, opA, nlines,
-                                      [&](int, int base, int k, T v) { W[base + k] = v; });
+// ====================================================================== sumfact3d
+//   S1 W1[l][m][k] = sum_n A[k][n] U[l][m][n]     (axis 2, P:440 / Fig. 2(b) P:213)
+//   S2 W2[l][j][k] = sum_m B[j][m] W1[l][m][k]    (axis 1, P:441 / P:214)
+//   S3 V [i][j][k] = sum_l C[i][l] W2[l][j][k]    (axis 0, P:442 / P:215; Fig. 2(d))
+// S1 and S2 run in place in the group buffer; S3 stores V straight from registers
+// (consecutive threads own consecutive (j,k): coalesced).
+template <int P1, typename T>
+__global__ void __launch_bounds__(Cfg<P1, P1, T, 2>::NT)
+sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, const T* __restrict__ C,
+                 const T* __restrict__ U, T* __restrict__ V) {
+    using CF = Cfg<P1, P1, T, 2>;
+    using G = Geo<P1, P1, T>;
+    constexpr int NT = CF::NT, R = CF::R;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T* opA = reinterpret_cast<T*>(smem_raw);
+    T* opB = opA + op_elems<P1, T>();
+    T* opC = opB + op_elems<P1, T>();
+    T* buf = opC + op_elems<P1, T>();
+    load_op<P1, T, NT>(opA, A);
+    load_op<P1, T, NT>(opB, B);
+    load_op<P1, T, NT>(opC, C);
+    group_loop_prefetch<P1, P1, T, NT, CF::E, CF::BUF>(N, U, buf, [&](T* in, int64_t e0, int ne) {
+        const int nlines = ne * P1 * P1;
+        apply_lines<P1, P1, 2, R, NT>(in, opA, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
         __syncthreads();
-        apply_lines<P1, P1, 1, R, NT>(W, opB, nlines,
-                                      [&](int, int base, int k, T v) { in[base + k * G::RS] = v; });
+        apply_lines<P1, P1, 1, R, NT>(in, opB, nlines, [&](int, int base, int k, T v) { in[base + k * G::RS] = v; });
         __syncthreads();
         T* Vg = V + e0 * G::NPTS;
         apply_lines<P1, P1, 0, R, NT>(in, opC, nlines, [&](int L, int, int k, T v) {
             st_cs(Vg + Line<P1, P1, 0, T>::gofs(L, k), v);
         });
-        cur ^= 1;
-    }
+    });
 }
 
 template <int P1, typename T>
 int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, cudaStream_t s) {
-    using CF = Cfg<P1, P1, T, 3>;
+    using CF = Cfg<P1, P1, T, 2>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
-    const int grid = grid_for(sumfact3d_kernel<P1, T>, CF::NT, CF::SMEM, ngroups, &occ);
-    sumfact3d_kernel<P1, T><<<grid, CF::NT, CF::SMEM, s>>>(N, A, B, C, U, V);
+    const size_t smem = CF::SMEM + op_elems<P1, T>() * sizeof(T);
+    const int grid = grid_for(sumfact3d_kernel<P1, T>, CF::NT, smem, ngroups, &occ);
+    sumfact3d_kernel<P1, T><<<grid, CF::NT, smem, s>>>(N, A, B, C, U, V);
     return launch_status();
 }
 
 // ====================================================================== sumfact2d
-//   W[l][j] = sum_m A[j][m] U[l][m]  (axis "2" = fastest);  V[i][j] = sum_l B[i][l] W[l][j]
+//   W[l][j] = sum_m A[j][m] U[l][m]  (rows, in place);  V[i][j] = sum_l B[i][l] W[l][j]
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, 1, double, 3>::NT)
+__global__ void __launch_bounds__(Cfg<P1, 1, double, 2>::NT)
 sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restrict__ B,
                  const double* __restrict__ U, double* __restrict__ V) {
     using T = double;
-    using CF = Cfg<P1, 1, T, 3>;
+    using CF = Cfg<P1, 1, T, 2>;
     using G = Geo<P1, 1, T>;
-    constexpr int E = CF::E, NT = CF::NT, R = CF::R;
+    constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* opA = reinterpret_cast<T*>(smem_raw);
     T* opB = opA + op_elems<P1, T>();
-    T* buf[2];
-    buf[0] = opB + op_elems<P1, T>();
-    buf[1] = buf[0] + CF::BUF;
-    T* W = buf[1] + CF::BUF;
+    T* buf = opB + op_elems<P1, T>();
     load_op<P1, T, NT>(opA, A);
     load_op<P1, T, NT>(opB, B);
-
-    const int64_t ngroups = (N + E - 1) / E;
-    int64_t g = blockIdx.x;
-    if (g < ngroups) load_group_async<P1, 1, T, NT>(buf[0], U + g * E * G::NPTS, imin64(E, N - g * E));
-    cp_async_commit();
-    int cur = 0;
-    for (; g < ngroups; g += gridDim.x) {
-        const int64_t e0 = g * E;
-        const int ne = imin64(E, N - e0);
+    group_loop_prefetch<P1, 1, T, NT, CF::E, CF::BUF>(N, U, buf, [&](T* in, int64_t e0, int ne) {
         const int nlines = ne * P1;
-        cp_async_wait_all();
-        __syncthreads();
-        T* in = buf[cur];
-        const int64_t gn = g + gridDim.x;
-        if (gn < ngroups)
-            load_group_async<P1, 1, T, NT>(buf[cur ^ 1], U + gn * E * G::NPTS, imin64(E, N - gn * E));
-        cp_async_commit();
-        apply_lines<P1, 1, 2, R, NT>(in, opA, nlines, [&](int, int base, int k, T v) { W[base + k] = v; });
+        apply_lines<P1, 1, 2, R, NT>(in, opA, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
         __syncthreads();
         T* Vg = V + e0 * G::NPTS;
-        apply_lines<P1, 1, 1, R, NT>(W, opB, nlines, [&](int L, int, int k, T v) {
+        apply_lines<P1, 1, 1, R, NT>(in, opB, nlines, [&](int L, int, int k, T v) {
             st_cs(Vg + Line<P1, 1, 1, T>::gofs(L, k), v);
         });
-        cur ^= 1;
-    }
+    });
 }
 
 template <int P1>
 int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* U, double* V, cudaStream_t s) {
-    using CF = Cfg<P1, 1, double, 3>;
+    using CF = Cfg<P1, 1, double, 2>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(sumfact2d_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
@@ -341,41 +330,23 @@ int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* 
 
 // ====================================================================== local_grad3
 //   ur = D along axis 2 (i), us = D along axis 1 (j), ut = D along axis 0 (k) of U[k][j][i]
+// us and ut are stored from registers (coalesced); ur is formed in place (its rows are
+// strided across threads) and copied out coalesced.
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, 3>::NT)
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 2>::NT)
 local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ U,
                    double* __restrict__ ur, double* __restrict__ us, double* __restrict__ ut) {
     using T = double;
-    using CF = Cfg<P1, P1, T, 3>;
+    using CF = Cfg<P1, P1, T, 2>;
     using G = Geo<P1, P1, T>;
-    constexpr int E = CF::E, NT = CF::NT, R = CF::R;
+    constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* opD = reinterpret_cast<T*>(smem_raw);
-    T* buf[2];
-    buf[0] = opD + op_elems<P1, T>();
-    buf[1] = buf[0] + CF::BUF;
-    T* W = buf[1] + CF::BUF;
+    T* buf = opD + 2 * op_elems<P1, T>();
     load_op<P1, T, NT>(opD, D);
-
-    const int64_t ngroups = (N + E - 1) / E;
-    int64_t g = blockIdx.x;
-    if (g < ngroups) load_group_async<P1, P1, T, NT>(buf[0], U + g * E * G::NPTS, imin64(E, N - g * E));
-    cp_async_commit();
-    int cur = 0;
-    for (; g < ngroups; g += gridDim.x) {
-        const int64_t e0 = g * E;
-        const int ne = imin64(E, N - e0);
+    group_loop_prefetch<P1, P1, T, NT, CF::E, CF::BUF>(N, U, buf, [&](T* in, int64_t e0, int ne) {
         const int nlines = ne * P1 * P1;
-        cp_async_wait_all();
-        __syncthreads();
-        T* in = buf[cur];
-        const int64_t gn = g + gridDim.x;
-        if (gn < ngroups)
-            load_group_async<P1, P1, T, NT>(buf[cur ^ 1], U + gn * E * G::NPTS, imin64(E, N - gn * E));
-        cp_async_commit();
         const int64_t gbase = e0 * G::NPTS;
-        // ur -> smem (its rows are strided across threads; stored coalesced below)
-        apply_lines<P1, P1, 2, R, NT>(in, opD, nlines, [&](int, int base, int k, T v) { W[base + k] = v; });
         apply_lines<P1, P1, 1, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
             st_cs(us + gbase + Line<P1, P1, 1, T>::gofs(L, k), v);
         });
@@ -383,16 +354,17 @@ local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __rest
             st_cs(ut + gbase + Line<P1, P1, 0, T>::gofs(L, k), v);
         });
         __syncthreads();
+        apply_lines<P1, P1, 2, R, NT>(in, opD, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
+        __syncthreads();
         const int total = ne * G::NPTS;
-        for (int f = threadIdx.x; f < total; f += NT) st_cs(ur + gbase + f, W[smem_index<P1, P1, T>(f)]);
-        cur ^= 1;
-    }
+        for (int f = threadIdx.x; f < total; f += NT) st_cs(ur + gbase + f, in[smem_index<P1, P1, T>(f)]);
+    });
 }
 
 template <int P1>
 int launch_local_grad3(int64_t N, const double* D, const double* U, double* ur, double* us, double* ut,
                        cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, 3>;
+    using CF = Cfg<P1, P1, double, 2>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(local_grad3_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
@@ -401,22 +373,21 @@ int launch_local_grad3(int64_t N, const double* D, const double* U, double* ur, 
 }
 
 // ====================================================================== local_grad3_t
-//   U = D^T along axis 2 of ur + D^T along axis 1 of us + D^T along axis 0 of ut
-//   (partial sums added in the order (r + s) + t)
+//   U = D^T along axis 2 of ur + D^T along axis 1 of us + D^T along axis 0 of ut,
+//   partial sums added in the order (r + s) + t.  Three field buffers, all in place.
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, 4>::NT)
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 3>::NT)
 local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ ur,
                      const double* __restrict__ us, const double* __restrict__ ut, double* __restrict__ U) {
     using T = double;
-    using CF = Cfg<P1, P1, T, 4>;
+    using CF = Cfg<P1, P1, T, 3>;
     using G = Geo<P1, P1, T>;
     constexpr int E = CF::E, NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* opT = reinterpret_cast<T*>(smem_raw);
-    T* bR = opT + op_elems<P1, T>();
+    T* bR = opT + 2 * op_elems<P1, T>();
     T* bS = bR + CF::BUF;
     T* bT = bS + CF::BUF;
-    T* W = bT + CF::BUF;
     load_op<P1, T, NT, true>(opT, D);
     const int64_t ngroups = (N + E - 1) / E;
     for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
@@ -431,13 +402,14 @@ local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __re
         cp_async_commit();
         cp_async_wait_all();
         __syncthreads();
-        apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { W[base + k] = v; });
+        apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
         __syncthreads();
-        apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines,
-                                      [&](int, int base, int k, T v) { W[base + k * G::RS] += v; });
+        apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines, [&](int, int base, int k, T v) {
+            bS[base + k * G::RS] = bR[base + k * G::RS] + v;
+        });
         __syncthreads();
         apply_lines<P1, P1, 0, R, NT>(bT, opT, nlines, [&](int L, int base, int k, T v) {
-            st_cs(U + gbase + Line<P1, P1, 0, T>::gofs(L, k), W[base + k * G::PS] + v);
+            st_cs(U + gbase + Line<P1, P1, 0, T>::gofs(L, k), bS[base + k * G::PS] + v);
         });
     }
 }
@@ -445,7 +417,7 @@ local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __re
 template <int P1>
 int launch_local_grad3_t(int64_t N, const double* D, const double* ur, const double* us, const double* ut,
                          double* U, cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, 4>;
+    using CF = Cfg<P1, P1, double, 3>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(local_grad3_t_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
@@ -454,19 +426,20 @@ int launch_local_grad3_t(int64_t N, const double* D, const double* ur, const dou
 }
 
 // ====================================================================== ax_e
+// (us, ut) from U into two buffers; ur in place over U; per-point geometric mixing in
+// place; then local_grad3_t in place as above.  Three field buffers.
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, 4>::NT)
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 3>::NT)
 ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ Uin,
             const double* __restrict__ Gm, double* __restrict__ Wout) {
     using T = double;
-    using CF = Cfg<P1, P1, T, 4>;
+    using CF = Cfg<P1, P1, T, 3>;
     using G = Geo<P1, P1, T>;
     constexpr int E = CF::E, NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* opD = reinterpret_cast<T*>(smem_raw);
     T* opT = opD + op_elems<P1, T>();
-    T* bU = opT + op_elems<P1, T>();
-    T* bR = bU + CF::BUF;
+    T* bR = opT + op_elems<P1, T>();  // holds U, then ur / wr
     T* bS = bR + CF::BUF;
     T* bT = bS + CF::BUF;
     load_op<P1, T, NT>(opD, D);
@@ -478,17 +451,17 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
         const int nlines = ne * P1 * P1;
         const int64_t gbase = e0 * G::NPTS;
         __syncthreads();
-        load_group_async<P1, P1, T, NT>(bU, Uin + gbase, ne);
+        load_group_async<P1, P1, T, NT>(bR, Uin + gbase, ne);
         cp_async_commit();
         cp_async_wait_all();
         __syncthreads();
-        apply_lines<P1, P1, 2, R, NT>(bU, opD, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
-        apply_lines<P1, P1, 1, R, NT>(bU, opD, nlines, [&](int, int base, int k, T v) { bS[base + k * G::RS] = v; });
-        apply_lines<P1, P1, 0, R, NT>(bU, opD, nlines, [&](int, int base, int k, T v) { bT[base + k * G::PS] = v; });
+        apply_lines<P1, P1, 1, R, NT>(bR, opD, nlines, [&](int, int base, int k, T v) { bS[base + k * G::RS] = v; });
+        apply_lines<P1, P1, 0, R, NT>(bR, opD, nlines, [&](int, int base, int k, T v) { bT[base + k * G::PS] = v; });
         __syncthreads();
-        // geometric mixing, one thread per point: G[e][c][q]
+        apply_lines<P1, P1, 2, R, NT>(bR, opD, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
+        __syncthreads();
         const int total = ne * G::NPTS;
-        for (int f = threadIdx.x; f < total; f += NT) {
+        for (int f = threadIdx.x; f < total; f += NT) {  // G[e][c][q]
             const int e = f / G::NPTS;
             const int q = f - e * G::NPTS;
             const T* gp = Gm + (e0 + e) * 6 * (int64_t)G::NPTS + q;
@@ -501,19 +474,21 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
             bT[si] = (g2 * r + g4 * s) + g5 * t;
         }
         __syncthreads();
-        apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { bU[base + k] = v; });
+        apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
         __syncthreads();
-        apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines, [&](int, int base, int k, T v) { bU[base + k * G::RS] += v; });
+        apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines, [&](int, int base, int k, T v) {
+            bS[base + k * G::RS] = bR[base + k * G::RS] + v;
+        });
         __syncthreads();
         apply_lines<P1, P1, 0, R, NT>(bT, opT, nlines, [&](int L, int base, int k, T v) {
-            st_cs(Wout + gbase + Line<P1, P1, 0, T>::gofs(L, k), bU[base + k * G::PS] + v);
+            st_cs(Wout + gbase + Line<P1, P1, 0, T>::gofs(L, k), bS[base + k * G::PS] + v);
         });
     }
 }
 
 template <int P1>
 int launch_ax_e(int64_t N, const double* D, const double* U, const double* Gm, double* W, cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, 4>;
+    using CF = Cfg<P1, P1, double, 3>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(ax_e_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
