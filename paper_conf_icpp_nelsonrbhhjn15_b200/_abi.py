@@ -9,7 +9,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbarracuda.so")
+LIB_PATH = os.environ.get("BARRACUDA_LIB") or os.path.join(_HERE, "libbarracuda.so")  # override: variant sweeps
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

@@ -23,6 +23,8 @@
 // positions.  The cube has odd strides (1, BS+1, (BS+1)^2) on every axis, so the flush is
 // bank-conflict free for any permutation.  The (h1,h2,h3) <-> storage-position maps are
 // derived here from the generating rule of DESIGN.md R12 (not copied from the oracle).
+#include <cstdlib>
+
 #include "common.cuh"
 
 namespace bc {
@@ -289,6 +291,209 @@ __global__ void __launch_bounds__(CcGeo<BS>::NT) ccsdt_kernel(const CcsdtParams 
     }
 }
 
+// ==================================================================================
+// Tensor-core path (BS = 16, d1/d2): FP64 DMMA mma.sync.m8n8k4 (no tcgen05 f64 kind
+// exists; DMMA reaches the full FP64 rate with 1/8 of DFMA's instruction count,
+// tools/fp64_peak.cu).  Same unit, cube accumulator and class flush as above.
+//   GEMM per variant: C[s][b] += A[s][k] * B[k][b], s = hole pair (256), b = third hole
+//   (16), k chunk KC = 8 (two m8n8k4 k-steps).  8 warps; warp w owns s in [32w, 32w+32)
+//   x all b: 4 x 2 fragments of 8x8 (16 fp64 accumulators per lane).
+//   smem operand layouts are chosen so fragment reads are bank-conflict free:
+//     d1: A = v2 slice stored [k][s] (row stride 260 = 4 mod 16), B = t2 slice [b][k] (12)
+//     d2: A = t2 slice stored [s][k] (row stride 12),             B = v2 slice [b][k] (12)
+//   and every staging copy is a 16-byte cp.async along the global-contiguous axis.
+// ==================================================================================
+template <int FAM>
+struct MmaGeo {
+    static constexpr int BS = 16, SD = 256, BD = 16, KC = 8, NT = 256;
+    static constexpr int NSTAGE = (FAM == FAM_D1) ? 3 : 2;  // keeps 2 CTAs per SM
+    static constexpr int SS_KS = 260;  // [k][s] row stride (d1 A)
+    static constexpr int SS_SK = 12;   // [s][k] row stride (d2 A)
+    static constexpr int SB_BK = 12;   // [b][k] row stride (B)
+    static constexpr int A_ELEMS = (FAM == FAM_D1) ? KC * SS_KS : SD * SS_SK;  // 2080 | 3072
+    static constexpr int B_ELEMS = BD * SB_BK;                                              // 192
+    static constexpr int STAGE = A_ELEMS + B_ELEMS;                                         // even
+    static constexpr int CST = BS + 1;
+    static constexpr int ACC = BS * CST * CST;  // 4624 (even): the stages stay 16B aligned
+    static constexpr size_t SMEM = (size_t)(ACC + NSTAGE * STAGE) * sizeof(double);
+};
+
+__device__ __forceinline__ void dmma_8x8x4(double& c0, double& c1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                 : "+d"(c0), "+d"(c1)
+                 : "d"(a), "d"(b));
+}
+
+__device__ __forceinline__ void cp_async_16_zfill(void* dst, const void* src, bool valid) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(smem_u32(dst)), "l"(src),
+                 "r"(valid ? 16 : 0));
+}
+template <int N>
+__device__ __forceinline__ void cp_async_wait_n() {
+    asm volatile("cp.async.wait_group %0;\n" ::"n"(N));
+}
+
+template <int FAM>
+__global__ void __launch_bounds__(256) ccsdt_mma_kernel(const CcsdtParams P) {
+    using MG = MmaGeo<FAM>;
+    constexpr int BS = MG::BS, KC = MG::KC, NT = MG::NT, CST = MG::CST;
+    extern __shared__ __align__(16) double sm[];
+    double* acc_s = sm;
+    double* stages = sm + MG::ACC;
+
+    const int ncubes = P.ncube[0] * P.ncube[1] * P.ncube[2];
+    const int cube = blockIdx.x % ncubes;
+    const int plane = blockIdx.x / ncubes;
+    int o[3], len[3];
+    o[0] = (cube % P.ncube[0]) * BS;
+    o[1] = ((cube / P.ncube[0]) % P.ncube[1]) * BS;
+    o[2] = (cube / (P.ncube[0] * P.ncube[1])) * BS;
+    for (int q = 0; q < 3; ++q) len[q] = min(BS, P.qe[q] - o[q]);
+    int qv[3];
+    qv[0] = plane % P.qe[3];
+    qv[1] = (plane / P.qe[3]) % P.qe[4];
+    qv[2] = plane / (P.qe[3] * P.qe[4]);
+    for (int i = threadIdx.x; i < BS * CST * CST; i += NT) acc_s[i] = 0.0;
+
+    const int H1 = P.ext[N_H1], H3 = P.ext[N_H3];
+    const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6];
+    const int K = P.ext[N_K];
+    const int nchunk = (K + KC - 1) / KC;
+    const int nstage = P.nentry * nchunk;
+
+    auto issue = [&](int st) {
+        double* A = stages + (st % MG::NSTAGE) * MG::STAGE;
+        double* B = A + MG::A_ELEMS;
+        const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+        const int c = P.ecls[e];
+        const int hp1 = P.hpos[c][0], hp2 = P.hpos[c][1], hp3 = P.hpos[c][2];
+        const int O1 = o[hp1], O2 = o[hp2], O3 = o[hp3];
+        const int L1 = len[hp1], L2 = len[hp2], L3 = len[hp3];
+        const int p4 = qv[P.ppos[e][0] - 3], p5 = qv[P.ppos[e][1] - 3], p6 = qv[P.ppos[e][2] - 3];
+        const double* __restrict__ t2 = P.opA[e];
+        const double* __restrict__ v2 = P.opB[e];
+        if constexpr (FAM == FAM_D1) {
+            const int H2 = P.ext[N_H2];
+            // A[k][s = i3 + 16 i2] = v2[h3, h2, p6, k]   (pairs along h3)
+            for (int x = threadIdx.x; x < KC * (BS * BS / 2); x += NT) {
+                const int kk = x >> 7, r = x & 127;
+                const int i2 = r >> 3, i3 = (r & 7) * 2;
+                const bool ok = (k0 + kk < K) && i3 < L3 && i2 < L2;
+                const int64_t off = ok ? (O3 + i3) + (int64_t)H3 * ((O2 + i2) + (int64_t)H2 * (p6 + (int64_t)P6 * (k0 + kk))) : 0;
+                cp_async_16_zfill(A + kk * MG::SS_KS + i3 + BS * i2, v2 + off, ok);
+            }
+            // B[b = i1][k] = t2[k, p4, p5, h1]   (pairs along k)
+            if (threadIdx.x < BS * KC / 2) {
+                const int i1 = threadIdx.x >> 2, kk = (threadIdx.x & 3) * 2;
+                const bool ok = (k0 + kk < K) && i1 < L1;
+                const int64_t off = ok ? (k0 + kk) + (int64_t)K * (p4 + (int64_t)P4 * (p5 + (int64_t)P5 * (O1 + i1))) : 0;
+                cp_async_16_zfill(B + i1 * MG::SB_BK + kk, t2 + off, ok);
+            }
+        } else {
+            // A[s = i1 + 16 i2][k] = t2[k, p4, h1, h2]   (pairs along k)
+            for (int x = threadIdx.x; x < BS * BS * (KC / 2); x += NT) {
+                const int sidx = x >> 2, kk = (x & 3) * 2;
+                const int i2 = sidx >> 4, i1 = sidx & 15;
+                const bool ok = (k0 + kk < K) && i1 < L1 && i2 < L2;
+                const int64_t off = ok ? (k0 + kk) + (int64_t)K * (p4 + (int64_t)P4 * ((O1 + i1) + (int64_t)H1 * (O2 + i2))) : 0;
+                cp_async_16_zfill(A + sidx * MG::SS_SK + kk, t2 + off, ok);
+            }
+            // B[b = i3][k] = v2[k, h3, p6, p5]   (pairs along k)
+            if (threadIdx.x < BS * KC / 2) {
+                const int i3 = threadIdx.x >> 2, kk = (threadIdx.x & 3) * 2;
+                const bool ok = (k0 + kk < K) && i3 < L3;
+                const int64_t off = ok ? (k0 + kk) + (int64_t)K * ((O3 + i3) + (int64_t)H3 * (p6 + (int64_t)P6 * p5)) : 0;
+                cp_async_16_zfill(B + i3 * MG::SB_BK + kk, v2 + off, ok);
+            }
+        }
+    };
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int gq = lane >> 2, tq = lane & 3;  // fragment group / thread-in-group
+    const int s_w = warp * 32;
+    double c[4][2][2];
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+        for (int ni = 0; ni < 2; ++ni) c[mi][ni][0] = c[mi][ni][1] = 0.0;
+
+    // prologue: NSTAGE-1 stages in flight
+#pragma unroll
+    for (int st = 0; st < MG::NSTAGE - 1; ++st) {
+        if (st < nstage) issue(st);
+        cp_async_commit();
+    }
+    for (int st = 0; st < nstage; ++st) {
+        cp_async_wait_n<MG::NSTAGE - 2>();  // stage st has landed (for this thread)
+        __syncthreads();                 // ... for all threads; stage st-1's buffer is free
+        if (st + MG::NSTAGE - 1 < nstage) issue(st + MG::NSTAGE - 1);
+        cp_async_commit();
+        const double* A = stages + (st % MG::NSTAGE) * MG::STAGE;
+        const double* B = A + MG::A_ELEMS;
+        const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+        const uint32_t smask = P.sign[e] < 0 ? 0x80000000u : 0u;
+#pragma unroll
+        for (int ks = 0; ks < KC / 4; ++ks) {
+            const int kk = ks * 4 + tq;
+            double bf[2], af[4];
+#pragma unroll
+            for (int ni = 0; ni < 2; ++ni) bf[ni] = flip_sign(B[(ni * 8 + gq) * MG::SB_BK + kk], smask);
+#pragma unroll
+            for (int mi = 0; mi < 4; ++mi) {
+                const int sidx = s_w + mi * 8 + gq;
+                af[mi] = (FAM == FAM_D1) ? A[kk * MG::SS_KS + sidx] : A[sidx * MG::SS_SK + kk];
+            }
+#pragma unroll
+            for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+                for (int ni = 0; ni < 2; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[mi], bf[ni]);
+        }
+        const bool last_chunk = (k0 + KC >= K);
+        if (last_chunk && (e + 1 == P.nentry || P.ecls[e + 1] != P.ecls[e])) {
+            const int cl = P.ecls[e];
+            const int strq[3] = {1, CST, CST * CST};
+            const int s1 = strq[P.hpos[cl][0]], s2 = strq[P.hpos[cl][1]], s3 = strq[P.hpos[cl][2]];
+#pragma unroll
+            for (int mi = 0; mi < 4; ++mi) {
+                const int sidx = s_w + mi * 8 + gq;
+                const int hi = sidx >> 4, lo = sidx & 15;
+                const int base = (FAM == FAM_D2) ? (lo * s1 + hi * s2) : (lo * s3 + hi * s2);
+                const int sb = (FAM == FAM_D2) ? s3 : s1;
+#pragma unroll
+                for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+                    for (int j = 0; j < 2; ++j) {
+                        acc_s[base + (ni * 8 + 2 * tq + j) * sb] += c[mi][ni][j];
+                        c[mi][ni][j] = 0.0;
+                    }
+            }
+        }
+    }
+    __syncthreads();
+    const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
+                          (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
+    const int nvol = len[0] * len[1] * len[2];
+    for (int i = threadIdx.x; i < nvol; i += NT) {
+        const int q0 = i % len[0], r = i / len[0];
+        const int q1 = r % len[1], q2 = r / len[1];
+        double* p = P.t3 + pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2));
+        *p += acc_s[q0 + CST * (q1 + CST * q2)];
+    }
+}
+
+template <int FAM>
+static int launch_ccsdt_mma(const CcsdtParams& P, cudaStream_t s) {
+    static bool init = false;
+    if (!init) {
+        cudaFuncSetAttribute(ccsdt_mma_kernel<FAM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)MmaGeo<FAM>::SMEM);
+        init = true;
+    }
+    const int64_t units = (int64_t)P.ncube[0] * P.ncube[1] * P.ncube[2] * P.qe[3] * P.qe[4] * P.qe[5];
+    if (units == 0) return BC_OK;
+    ccsdt_mma_kernel<FAM><<<(unsigned)units, MmaGeo<FAM>::NT, MmaGeo<FAM>::SMEM, s>>>(P);
+    return launch_status();
+}
+
 // ------------------------------------------------------------------------------------ host
 static int choose_bs(const int* qe) {
     // smallest padded volume over the three hole positions; ties -> larger cube
@@ -352,6 +557,11 @@ int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const
     P.ncls = ncls;
     const int bs = choose_bs(P.qe);
     for (int q = 0; q < 3; ++q) P.ncube[q] = (P.qe[q] + bs - 1) / bs;
+    // tensor-core path: 16-cubes with 16-byte-aligned operand pairs (even k, even h3 for d1)
+    const bool mma_ok = bs == 16 && (ext7[N_K] % 2 == 0) && (fam != FAM_D1 || ext7[N_H3] % 2 == 0) &&
+                        getenv("BC_NO_MMA") == nullptr;
+    if (mma_ok && fam == FAM_D1) return launch_ccsdt_mma<FAM_D1>(P, s);
+    if (mma_ok && fam == FAM_D2) return launch_ccsdt_mma<FAM_D2>(P, s);
 #define LAUNCH(F)                                                          \
     if (bs == 16) return launch_ccsdt_bs<F, 16>(P, s);                      \
     if (bs == 12) return launch_ccsdt_bs<F, 12>(P, s);                      \

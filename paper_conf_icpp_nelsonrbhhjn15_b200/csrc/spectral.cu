@@ -198,10 +198,16 @@ __host__ __device__ __forceinline__ int imin64(int64_t a, int64_t b) { return (i
 template <int P1, int NA, typename T, int NBUF>
 struct Cfg {
     using G = Geo<P1, NA, T>;
-    static constexpr int BUF_BYTES = 36 * 1024;  // target bytes per element-group buffer
+#ifndef BC_SPEC_BUF_KB
+#define BC_SPEC_BUF_KB 36
+#endif
+#ifndef BC_SPEC_R
+#define BC_SPEC_R 2
+#endif
+    static constexpr int BUF_BYTES = BC_SPEC_BUF_KB * 1024;  // target bytes per element-group buffer
     static constexpr int E0 = BUF_BYTES / (G::ES * (int)sizeof(T));
     static constexpr int E = E0 < 2 ? 1 : (E0 & ~1);  // even: groups of odd-P1 elements stay 16B-aligned
-    static constexpr int R = 2;
+    static constexpr int R = BC_SPEC_R;
     static constexpr int LINES = E * NA * P1;  // lines per axis per group (E * NPTS / P1)
     static constexpr int NT0 = ((LINES + R - 1) / R + 31) / 32 * 32;
     static constexpr int NT = NT0 < 64 ? 64 : (NT0 > 512 ? 512 : NT0);
