@@ -361,49 +361,79 @@ __global__ void __launch_bounds__(256) ccsdt_mma_kernel(const CcsdtParams P) {
     const int nchunk = (K + KC - 1) / KC;
     const int nstage = P.nentry * nchunk;
 
+    // ---- per-thread staging plan.  Thread copies 16-byte pairs at fixed hole positions:
+    //   d1 A: (i2, i3) = ((t & 127) >> 3, 2 (t & 7)), k = (t >> 7) + 2 j      (j < 4)
+    //   d2 A: (i1, i2) = ((t >> 2) & 15, (t >> 6) + 4 j), k pair 2 (t & 3)      (j < 4)
+    //   B (t < 64): third hole i = t >> 2, k pair 2 (t & 3)
+    // Hole offsets are computed once per class; a variant adds its particle offset and a
+    // stage its k offset, so each copy is a pointer increment.
+    const int tid = threadIdx.x;
+    const int H2 = P.ext[N_H2];
+    int64_t hA[3][4];      // per class: hole part of the A offsets (or -1: outside the block)
+    int64_t hB[3];
+    for (int c = 0; c < P.ncls; ++c) {
+        const int hp1 = P.hpos[c][0], hp2 = P.hpos[c][1], hp3 = P.hpos[c][2];
+        const int O1 = o[hp1], O2 = o[hp2], O3 = o[hp3];
+        const int L1 = len[hp1], L2 = len[hp2], L3 = len[hp3];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            if constexpr (FAM == FAM_D1) {
+                const int i2 = (tid & 127) >> 3, i3 = (tid & 7) * 2;
+                hA[c][j] = (i3 < L3 && i2 < L2) ? (O3 + i3) + (int64_t)H3 * (O2 + i2) : -1;
+            } else {
+                const int i1 = (tid >> 2) & 15, i2 = (tid >> 6) + 4 * j;
+                hA[c][j] = (i1 < L1 && i2 < L2) ? (int64_t)K * P4 * ((O1 + i1) + (int64_t)H1 * (O2 + i2)) : -1;
+            }
+        }
+        const int ib = tid >> 2;
+        if constexpr (FAM == FAM_D1)
+            hB[c] = (tid < 64 && ib < L1) ? (int64_t)K * P4 * P5 * (O1 + ib) : -1;
+        else
+            hB[c] = (tid < 64 && ib < L3) ? (int64_t)K * (O3 + ib) : -1;
+    }
+    const int kA = (FAM == FAM_D1) ? (tid >> 7) : 2 * (tid & 3);  // k offset of A copy j = 0
+    const int kB = 2 * (tid & 3);
+    const int dstA = (FAM == FAM_D1) ? (tid >> 7) * MG::SS_KS + 2 * (tid & 127)  // s = i3 + 16 i2 = 2 (t & 127)
+                                     : (tid >> 2) * MG::SS_SK + 2 * (tid & 3);
+    const int dstB = (tid >> 2) * MG::SB_BK + 2 * (tid & 3);
+
     auto issue = [&](int st) {
         double* A = stages + (st % MG::NSTAGE) * MG::STAGE;
         double* B = A + MG::A_ELEMS;
         const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
         const int c = P.ecls[e];
-        const int hp1 = P.hpos[c][0], hp2 = P.hpos[c][1], hp3 = P.hpos[c][2];
-        const int O1 = o[hp1], O2 = o[hp2], O3 = o[hp3];
-        const int L1 = len[hp1], L2 = len[hp2], L3 = len[hp3];
         const int p4 = qv[P.ppos[e][0] - 3], p5 = qv[P.ppos[e][1] - 3], p6 = qv[P.ppos[e][2] - 3];
         const double* __restrict__ t2 = P.opA[e];
         const double* __restrict__ v2 = P.opB[e];
         if constexpr (FAM == FAM_D1) {
-            const int H2 = P.ext[N_H2];
-            // A[k][s = i3 + 16 i2] = v2[h3, h2, p6, k]   (pairs along h3)
-            for (int x = threadIdx.x; x < KC * (BS * BS / 2); x += NT) {
-                const int kk = x >> 7, r = x & 127;
-                const int i2 = r >> 3, i3 = (r & 7) * 2;
-                const bool ok = (k0 + kk < K) && i3 < L3 && i2 < L2;
-                const int64_t off = ok ? (O3 + i3) + (int64_t)H3 * ((O2 + i2) + (int64_t)H2 * (p6 + (int64_t)P6 * (k0 + kk))) : 0;
-                cp_async_16_zfill(A + kk * MG::SS_KS + i3 + BS * i2, v2 + off, ok);
+            // A[k][s] = v2[h3, h2, p6, k]: offset hole + H3 H2 (p6 + P6 k)
+            const int64_t sk = (int64_t)H3 * H2 * P6;
+            const double* base = v2 + (int64_t)H3 * H2 * p6 + sk * (k0 + kA);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const bool ok = hA[c][j] >= 0 && (k0 + kA + 2 * j) < K;
+                cp_async_16_zfill(A + dstA + 2 * j * MG::SS_KS, base + (ok ? hA[c][j] + 2 * j * sk : 0), ok);
             }
-            // B[b = i1][k] = t2[k, p4, p5, h1]   (pairs along k)
-            if (threadIdx.x < BS * KC / 2) {
-                const int i1 = threadIdx.x >> 2, kk = (threadIdx.x & 3) * 2;
-                const bool ok = (k0 + kk < K) && i1 < L1;
-                const int64_t off = ok ? (k0 + kk) + (int64_t)K * (p4 + (int64_t)P4 * (p5 + (int64_t)P5 * (O1 + i1))) : 0;
-                cp_async_16_zfill(B + i1 * MG::SB_BK + kk, t2 + off, ok);
+            // B[b][k] = t2[k, p4, p5, h1]: offset k + K (p4 + P4 p5) + hole
+            if (tid < 64) {
+                const bool ok = hB[c] >= 0 && (k0 + kB) < K;
+                const double* src = t2 + (ok ? hB[c] + (k0 + kB) + (int64_t)K * (p4 + (int64_t)P4 * p5) : 0);
+                cp_async_16_zfill(B + dstB, src, ok);
             }
         } else {
-            // A[s = i1 + 16 i2][k] = t2[k, p4, h1, h2]   (pairs along k)
-            for (int x = threadIdx.x; x < BS * BS * (KC / 2); x += NT) {
-                const int sidx = x >> 2, kk = (x & 3) * 2;
-                const int i2 = sidx >> 4, i1 = sidx & 15;
-                const bool ok = (k0 + kk < K) && i1 < L1 && i2 < L2;
-                const int64_t off = ok ? (k0 + kk) + (int64_t)K * (p4 + (int64_t)P4 * ((O1 + i1) + (int64_t)H1 * (O2 + i2))) : 0;
-                cp_async_16_zfill(A + sidx * MG::SS_SK + kk, t2 + off, ok);
+            // A[s][k] = t2[k, p4, h1, h2]: offset k + K p4 + hole
+            const double* base = t2 + (k0 + kA) + (int64_t)K * p4;
+            const bool kok = (k0 + kA) < K;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const bool ok = kok && hA[c][j] >= 0;
+                cp_async_16_zfill(A + dstA + 64 * j * MG::SS_SK, base + (ok ? hA[c][j] : 0), ok);
             }
-            // B[b = i3][k] = v2[k, h3, p6, p5]   (pairs along k)
-            if (threadIdx.x < BS * KC / 2) {
-                const int i3 = threadIdx.x >> 2, kk = (threadIdx.x & 3) * 2;
-                const bool ok = (k0 + kk < K) && i3 < L3;
-                const int64_t off = ok ? (k0 + kk) + (int64_t)K * ((O3 + i3) + (int64_t)H3 * (p6 + (int64_t)P6 * p5)) : 0;
-                cp_async_16_zfill(B + i3 * MG::SB_BK + kk, v2 + off, ok);
+            // B[b][k] = v2[k, h3, p6, p5]: offset k + K (h3 + H3 (p6 + P6 p5))
+            if (tid < 64) {
+                const bool ok = hB[c] >= 0 && (k0 + kB) < K;
+                const double* src = v2 + (ok ? hB[c] + (k0 + kB) + (int64_t)K * H3 * (p6 + (int64_t)P6 * p5) : 0);
+                cp_async_16_zfill(B + dstB, src, ok);
             }
         }
     };
