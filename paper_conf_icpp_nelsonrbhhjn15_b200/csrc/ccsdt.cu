@@ -23,7 +23,11 @@
 // positions.  The cube has odd strides (1, BS+1, (BS+1)^2) on every axis, so the flush is
 // bank-conflict free for any permutation.  The (h1,h2,h3) <-> storage-position maps are
 // derived here from the generating rule of DESIGN.md R12 (not copied from the oracle).
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
 #include <cstdlib>
+#include <cstring>
 
 #include "common.cuh"
 
@@ -353,7 +357,18 @@ __global__ void __launch_bounds__(256) ccsdt_mma_kernel(const CcsdtParams P) {
     qv[0] = plane % P.qe[3];
     qv[1] = (plane / P.qe[3]) % P.qe[4];
     qv[2] = plane / (P.qe[3] * P.qe[4]);
-    for (int i = threadIdx.x; i < BS * CST * CST; i += NT) acc_s[i] = 0.0;
+    // the unit's t3 values seed the accumulator cube (read once, asynchronously, while
+    // the first operand stages stream in); the cube is stored back once at the end
+    const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
+                          (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
+    const int nvol = len[0] * len[1] * len[2];
+    for (int i = threadIdx.x; i < nvol; i += NT) {
+        const int q0 = i % len[0], r = i / len[0];
+        const int q1 = r % len[1], q2 = r / len[1];
+        cp_async_8(acc_s + q0 + CST * (q1 + CST * q2),
+                   P.t3 + pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2)));
+    }
+    cp_async_commit();
 
     const int H1 = P.ext[N_H1], H3 = P.ext[N_H3];
     const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6];
@@ -402,7 +417,8 @@ __global__ void __launch_bounds__(256) ccsdt_mma_kernel(const CcsdtParams P) {
         double* B = A + MG::A_ELEMS;
         const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
         const int c = P.ecls[e];
-        const int p4 = qv[P.ppos[e][0] - 3], p5 = qv[P.ppos[e][1] - 3], p6 = qv[P.ppos[e][2] - 3];
+        auto pick = [&](int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
+        const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
         const double* __restrict__ t2 = P.opA[e];
         const double* __restrict__ v2 = P.opB[e];
         if constexpr (FAM == FAM_D1) {
@@ -499,15 +515,13 @@ __global__ void __launch_bounds__(256) ccsdt_mma_kernel(const CcsdtParams P) {
             }
         }
     }
+    cp_async_wait_all();  // (only matters when nstage == 0)
     __syncthreads();
-    const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
-                          (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
-    const int nvol = len[0] * len[1] * len[2];
     for (int i = threadIdx.x; i < nvol; i += NT) {
         const int q0 = i % len[0], r = i / len[0];
         const int q1 = r % len[1], q2 = r / len[1];
-        double* p = P.t3 + pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2));
-        *p += acc_s[q0 + CST * (q1 + CST * q2)];
+        P.t3[pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2))] =
+            acc_s[q0 + CST * (q1 + CST * q2)];
     }
 }
 
@@ -521,6 +535,315 @@ static int launch_ccsdt_mma(const CcsdtParams& P, cudaStream_t s) {
     const int64_t units = (int64_t)P.ncube[0] * P.ncube[1] * P.ncube[2] * P.qe[3] * P.qe[4] * P.qe[5];
     if (units == 0) return BC_OK;
     ccsdt_mma_kernel<FAM><<<(unsigned)units, MmaGeo<FAM>::NT, MmaGeo<FAM>::SMEM, s>>>(P);
+    return launch_status();
+}
+
+// ==================================================================================
+// Blackwell-native path (BS = 16, d1/d2): persistent, warp-specialised kernel.
+//   warp 8 (producer): one lane drives the Tensor Memory Accelerator —
+//     cp.async.bulk.tensor copies of each (variant, k-chunk) operand slice straight from
+//     the 4-D t2 / v2 tensors into a 4-deep shared-memory ring, with hardware swizzling
+//     (bank-conflict-free fragment reads) and out-of-bounds zero fill (ragged blocks),
+//     completion tracked by full/empty mbarriers — no per-thread staging code at all.
+//   warps 0-7 (consumers): FP64 DMMA m8n8k4 on the staged slices, accumulating per hole
+//     permutation class in registers, flushed into the unit's t3 cube in shared memory.
+// Each CTA loops over units (a 16^3 hole cube x one particle plane); the unit's t3 values
+// seed the cube (read once, cp.async) and the cube is stored once.
+// Operand layouts in one stage (KC = 8 k values):
+//   d1: A = v2[h3, O2+i2, p6, k] for i2 < 16: 16 copies of [k][h3] (128 B rows, 128B swizzle)
+//       B = t2[k, p4, p5, h1]: [h1][k] (64 B rows, 64B swizzle)
+//   d2: A = t2[k, p4, h1, h2]: [h2][h1][k] (64 B rows, 64B swizzle)
+//       B = v2[k, h3, p6, p5]: [h3][k] (64 B rows, 64B swizzle)
+// Fragment rows are permuted ({0,1,8,9,2,3,10,11} for the 128B case, {0,1,4,5,2,3,6,7}
+// for the 64B case) so that each half-warp touches 16 distinct banks.
+// ==================================================================================
+struct TmaMaps {
+    CUtensorMap a[9];  // d1: v2_v (h3,h2,p6,k) | d2: t2_v (k,p4,h1,h2)
+    CUtensorMap b[9];  // d1: t2_v (k,p4,p5,h1) | d2: v2_v (k,h3,p6,p5)
+};
+
+struct TmaGeo {
+    static constexpr int BS = 16, KC = 8, NS = 4, NCW = 8, NT = (NCW + 1) * 32;
+    static constexpr int A_BYTES = 16 * 16 * KC * 8;  // 16 KiB
+    static constexpr int B_BYTES = 16 * KC * 8;       // 1 KiB
+    static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;  // 17 KiB (multiple of 1 KiB)
+    static constexpr int CST = BS + 1;
+    static constexpr int ACC = BS * CST * CST;          // doubles
+    static constexpr size_t SMEM = 1024 + (size_t)NS * STAGE_BYTES + ACC * 8 + 2 * NS * 8;
+};
+
+__device__ __forceinline__ void mbar_init(uint32_t bar, int count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(bar), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, int bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, int parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n}\n" ::"r"(bar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void tma_load_4d(uint32_t dst, const CUtensorMap* map, int c0, int c1, int c2, int c3,
+                                            uint32_t bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], [%6];\n"
+        ::"r"(dst), "l"(map), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void named_bar_sync(int id, int n) {
+    asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(n) : "memory");
+}
+
+// fragment row permutations (see header)
+__device__ __forceinline__ int perm128(int g) { return (g & 1) + 8 * ((g >> 1) & 1) + 2 * (g >> 2); }
+__device__ __forceinline__ int perm64(int g) { return (g & 1) + 4 * ((g >> 1) & 1) + 2 * (g >> 2); }
+// byte offset of element (row, col) in 64-byte rows under the 64B swizzle
+__device__ __forceinline__ uint32_t swz64(uint32_t row, uint32_t col) {
+    const uint32_t off = row * 64 + col * 8;
+    return off ^ (((off >> 7) & 3) << 4);
+}
+
+template <int FAM>
+__global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_constant__ CcsdtParams P,
+                                                               const __grid_constant__ TmaMaps M, int units) {
+    using TG = TmaGeo;
+    constexpr int BS = TG::BS, KC = TG::KC, NS = TG::NS, CST = TG::CST;
+    extern __shared__ unsigned char smem_raw[];
+    const uint32_t raw = smem_u32(smem_raw);
+    const uint32_t base = (raw + 1023) & ~1023u;
+    unsigned char* gbase = smem_raw + (base - raw);
+    const uint32_t st_u32 = base;                                   // stage ring
+    double* acc_s = reinterpret_cast<double*>(gbase + NS * TG::STAGE_BYTES);
+    const uint32_t bar_full = base + NS * TG::STAGE_BYTES + TG::ACC * 8;
+    const uint32_t bar_empty = bar_full + NS * 8;
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < NS; ++i) {
+            mbar_init(bar_full + 8 * i, 1);
+            mbar_init(bar_empty + 8 * i, TG::NCW);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    __syncthreads();
+
+    const int ncubes = P.ncube[0] * P.ncube[1] * P.ncube[2];
+    const int K = P.ext[N_K];
+    const int nchunk = (K + KC - 1) / KC;
+    const int nstage = P.nentry * nchunk;
+
+    auto decode = [&](int u, int* o, int* len, int* qv) {
+        const int cube = u % ncubes, plane = u / ncubes;
+        o[0] = (cube % P.ncube[0]) * BS;
+        o[1] = ((cube / P.ncube[0]) % P.ncube[1]) * BS;
+        o[2] = (cube / (P.ncube[0] * P.ncube[1])) * BS;
+        for (int q = 0; q < 3; ++q) len[q] = min(BS, P.qe[q] - o[q]);
+        qv[0] = plane % P.qe[3];
+        qv[1] = (plane / P.qe[3]) % P.qe[4];
+        qv[2] = plane / (P.qe[3] * P.qe[4]);
+    };
+
+    if (warp == TG::NCW) {
+        // ================================ producer
+        if (lane == 0) {
+            int g = 0;
+            for (int u = blockIdx.x; u < units; u += gridDim.x) {
+                int o[3], len[3], qv[3];
+                decode(u, o, len, qv);
+                for (int st = 0; st < nstage; ++st, ++g) {
+                    const int slot = g % NS;
+                    mbar_wait(bar_empty + 8 * slot, ((g / NS) & 1) ^ 1);
+                    const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+                    const int c = P.ecls[e];
+                    const int O1 = o[P.hpos[c][0]], O2 = o[P.hpos[c][1]], O3 = o[P.hpos[c][2]];
+                    auto pick = [&](int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
+                    const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
+                    const uint32_t full = bar_full + 8 * slot;
+                    const uint32_t A = st_u32 + slot * TG::STAGE_BYTES;
+                    const uint32_t B = A + TG::A_BYTES;
+                    mbar_expect_tx(full, TG::STAGE_BYTES);
+                    if constexpr (FAM == FAM_D1) {
+#pragma unroll 1
+                        for (int i2 = 0; i2 < 16; ++i2) tma_load_4d(A + i2 * 1024, &M.a[e], O3, O2 + i2, p6, k0, full);
+                        tma_load_4d(B, &M.b[e], k0, p4, p5, O1, full);
+                    } else {
+                        tma_load_4d(A, &M.a[e], k0, p4, O1, O2, full);
+                        tma_load_4d(B, &M.b[e], k0, O3, p6, p5, full);
+                    }
+                }
+            }
+        }
+        return;
+    }
+
+    // ==================================== consumers (warps 0..7)
+    const int gq = lane >> 2, tq = lane & 3;
+    const int tid = threadIdx.x;  // < 256
+    int g = 0;
+    for (int u = blockIdx.x; u < units; u += gridDim.x) {
+        int o[3], len[3], qv[3];
+        decode(u, o, len, qv);
+        const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
+                              (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
+        const int nvol = len[0] * len[1] * len[2];
+        for (int i = tid; i < nvol; i += 256) {
+            const int q0 = i % len[0], r = i / len[0];
+            const int q1 = r % len[1], q2 = r / len[1];
+            cp_async_8(acc_s + q0 + CST * (q1 + CST * q2),
+                       P.t3 + pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2)));
+        }
+        cp_async_commit();
+        cp_async_wait_all();
+        named_bar_sync(1, 256);
+
+        double c[4][2][2];
+#pragma unroll
+        for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+            for (int ni = 0; ni < 2; ++ni) c[mi][ni][0] = c[mi][ni][1] = 0.0;
+
+        for (int st = 0; st < nstage; ++st, ++g) {
+            const int slot = g % NS;
+            mbar_wait(bar_full + 8 * slot, (g / NS) & 1);
+            const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
+            const unsigned char* B = A + TG::A_BYTES;
+            const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+            const uint32_t smask = P.sign[e] < 0 ? 0x80000000u : 0u;
+#pragma unroll
+            for (int ks = 0; ks < KC / 4; ++ks) {
+                const int kk = ks * 4 + tq;
+                double bf[2], af[4];
+#pragma unroll
+                for (int ni = 0; ni < 2; ++ni)
+                    bf[ni] = flip_sign(*reinterpret_cast<const double*>(B + swz64(ni * 8 + perm64(gq), kk)), smask);
+#pragma unroll
+                for (int mi = 0; mi < 4; ++mi) {
+                    uint32_t off;
+                    if constexpr (FAM == FAM_D1) {
+                        const int i2 = 2 * warp + (mi >> 1);
+                        const int i3 = perm128(gq) + 4 * (mi & 1);
+                        off = i2 * 1024 + kk * 128 + ((((i3 >> 1) ^ kk) & 7) << 4) + ((i3 & 1) << 3);
+                    } else {
+                        off = swz64(32 * warp + 8 * mi + perm64(gq), kk);
+                    }
+                    af[mi] = *reinterpret_cast<const double*>(A + off);
+                }
+#pragma unroll
+                for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+                    for (int ni = 0; ni < 2; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[mi], bf[ni]);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
+            const bool last_chunk = (k0 + KC >= K);
+            if (last_chunk && (e + 1 == P.nentry || P.ecls[e + 1] != P.ecls[e])) {
+                const int cl = P.ecls[e];
+                const int h1p = P.hpos[cl][0], h2p = P.hpos[cl][1], h3p = P.hpos[cl][2];
+                const int s1 = h1p == 0 ? 1 : (h1p == 1 ? CST : CST * CST);
+                const int s2 = h2p == 0 ? 1 : (h2p == 1 ? CST : CST * CST);
+                const int s3 = h3p == 0 ? 1 : (h3p == 1 ? CST : CST * CST);
+#pragma unroll
+                for (int mi = 0; mi < 4; ++mi) {
+                    int hi, lo;  // strided pair (lo = fast name, hi = h2)
+                    if constexpr (FAM == FAM_D1) {
+                        hi = 2 * warp + (mi >> 1);
+                        lo = perm128(gq) + 4 * (mi & 1);
+                    } else {
+                        const int sidx = 32 * warp + 8 * mi + perm64(gq);
+                        hi = sidx >> 4;
+                        lo = sidx & 15;
+                    }
+                    const int rowoff = (FAM == FAM_D2) ? (lo * s1 + hi * s2) : (lo * s3 + hi * s2);
+                    const int sb = (FAM == FAM_D2) ? s3 : s1;
+#pragma unroll
+                    for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+                        for (int j = 0; j < 2; ++j) {
+                            acc_s[rowoff + (ni * 8 + perm64(2 * tq + j)) * sb] += c[mi][ni][j];
+                            c[mi][ni][j] = 0.0;
+                        }
+                }
+            }
+        }
+        named_bar_sync(1, 256);
+        for (int i = tid; i < nvol; i += 256) {
+            const int q0 = i % len[0], r = i / len[0];
+            const int q1 = r % len[1], q2 = r / len[1];
+            P.t3[pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2))] =
+                acc_s[q0 + CST * (q1 + CST * q2)];
+        }
+        named_bar_sync(1, 256);
+    }
+}
+
+// ---- host: tensor maps (driver entry point, no -lcuda)
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static bool tried = false;
+    if (!tried) {
+        tried = true;
+        void* f = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
+    }
+    return fn;
+}
+
+static bool encode_4d(CUtensorMap* m, const double* ptr, const int* dims, const int* box, bool swz128) {
+    auto enc = get_encode();
+    if (!enc) return false;
+    cuuint64_t gdim[4], gstr[3];
+    cuuint32_t bdim[4], estr[4] = {1, 1, 1, 1};
+    cuuint64_t st = 8;
+    for (int i = 0; i < 4; ++i) {
+        gdim[i] = (cuuint64_t)dims[i];
+        bdim[i] = (cuuint32_t)box[i];
+        if (i > 0) gstr[i - 1] = st;
+        st *= (cuuint64_t)dims[i];
+    }
+    const CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<double*>(ptr), gdim, gstr, bdim, estr,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, swz128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
+                           CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
+// returns -1 when the TMA path is unavailable (caller falls back)
+template <int FAM>
+static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
+    TmaMaps M;
+    memset(&M, 0, sizeof(M));
+    const int H1 = P.ext[N_H1], H2 = P.ext[N_H2], H3 = P.ext[N_H3];
+    const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6], K = P.ext[N_K];
+    for (int e = 0; e < P.nentry; ++e) {
+        bool ok;
+        if (FAM == FAM_D1) {
+            const int da[4] = {H3, H2, P6, K}, ba[4] = {16, 1, 1, TmaGeo::KC};
+            const int db[4] = {K, P4, P5, H1}, bb[4] = {TmaGeo::KC, 1, 1, 16};
+            ok = encode_4d(&M.a[e], P.opB[e], da, ba, true) && encode_4d(&M.b[e], P.opA[e], db, bb, false);
+        } else {
+            const int da[4] = {K, P4, H1, H2}, ba[4] = {TmaGeo::KC, 1, 16, 16};
+            const int db[4] = {K, H3, P6, P5}, bb[4] = {TmaGeo::KC, 16, 1, 1};
+            ok = encode_4d(&M.a[e], P.opA[e], da, ba, false) && encode_4d(&M.b[e], P.opB[e], db, bb, false);
+        }
+        if (!ok) return -1;
+    }
+    static int occ = 0;
+    if (occ == 0) {
+        cudaFuncSetAttribute(ccsdt_tma_kernel<FAM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TmaGeo::SMEM);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_tma_kernel<FAM>, TmaGeo::NT, TmaGeo::SMEM);
+        if (occ < 1) occ = 1;
+    }
+    const int64_t units = (int64_t)P.ncube[0] * P.ncube[1] * P.ncube[2] * P.qe[3] * P.qe[4] * P.qe[5];
+    if (units == 0) return BC_OK;
+    const int64_t cap = (int64_t)num_sms() * occ;
+    const int grid = (int)(units < cap ? units : cap);
+    ccsdt_tma_kernel<FAM><<<grid, TmaGeo::NT, TmaGeo::SMEM, s>>>(P, M, (int)units);
     return launch_status();
 }
 
@@ -590,6 +913,11 @@ int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const
     // tensor-core path: 16-cubes with 16-byte-aligned operand pairs (even k, even h3 for d1)
     const bool mma_ok = bs == 16 && (ext7[N_K] % 2 == 0) && (fam != FAM_D1 || ext7[N_H3] % 2 == 0) &&
                         getenv("BC_NO_MMA") == nullptr;
+    const bool tma_ok = mma_ok && getenv("BC_NO_TMA") == nullptr;
+    if (tma_ok) {
+        const int st = (fam == FAM_D1) ? launch_ccsdt_tma<FAM_D1>(P, s) : (fam == FAM_D2 ? launch_ccsdt_tma<FAM_D2>(P, s) : -1);
+        if (st != -1) return st;
+    }
     if (mma_ok && fam == FAM_D1) return launch_ccsdt_mma<FAM_D1>(P, s);
     if (mma_ok && fam == FAM_D2) return launch_ccsdt_mma<FAM_D2>(P, s);
 #define LAUNCH(F)                                                          \
