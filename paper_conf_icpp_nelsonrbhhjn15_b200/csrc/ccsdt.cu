@@ -563,6 +563,7 @@ struct TmaMaps {
 };
 
 struct TmaGeo {
+    // two CTAs per SM (measured better than one CTA with a deeper ring), 4-deep ring
     static constexpr int BS = 16, KC = 8, NS = 4, NCW = 8, NT = (NCW + 1) * 32;
     static constexpr int A_BYTES = 16 * 16 * KC * 8;  // 16 KiB
     static constexpr int B_BYTES = 16 * KC * 8;       // 1 KiB
@@ -648,32 +649,35 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
     };
 
     if (warp == TG::NCW) {
-        // ================================ producer
-        if (lane == 0) {
-            int g = 0;
-            for (int u = blockIdx.x; u < units; u += gridDim.x) {
-                int o[3], len[3], qv[3];
-                decode(u, o, len, qv);
-                for (int st = 0; st < nstage; ++st, ++g) {
-                    const int slot = g % NS;
+        // ================================ producer: lane 0 arms the stage, lanes issue copies
+        int g = 0;
+        for (int u = blockIdx.x; u < units; u += gridDim.x) {
+            int o[3], len[3], qv[3];
+            decode(u, o, len, qv);
+            for (int st = 0; st < nstage; ++st, ++g) {
+                const int slot = g % NS;
+                const uint32_t full = bar_full + 8 * slot;
+                if (lane == 0) {
                     mbar_wait(bar_empty + 8 * slot, ((g / NS) & 1) ^ 1);
-                    const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
-                    const int c = P.ecls[e];
-                    const int O1 = o[P.hpos[c][0]], O2 = o[P.hpos[c][1]], O3 = o[P.hpos[c][2]];
-                    auto pick = [&](int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
-                    const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
-                    const uint32_t full = bar_full + 8 * slot;
-                    const uint32_t A = st_u32 + slot * TG::STAGE_BYTES;
-                    const uint32_t B = A + TG::A_BYTES;
                     mbar_expect_tx(full, TG::STAGE_BYTES);
-                    if constexpr (FAM == FAM_D1) {
+                }
+                __syncwarp();
+                const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+                const int c = P.ecls[e];
+                const int O1 = o[P.hpos[c][0]], O2 = o[P.hpos[c][1]], O3 = o[P.hpos[c][2]];
+                auto pick = [&](int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
+                const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
+                const uint32_t A = st_u32 + slot * TG::STAGE_BYTES;
+                const uint32_t B = A + TG::A_BYTES;
+                if constexpr (FAM == FAM_D1) {
+                    if (lane == 0) {  // one issuing lane measured faster than spreading the 17 copies
 #pragma unroll 1
                         for (int i2 = 0; i2 < 16; ++i2) tma_load_4d(A + i2 * 1024, &M.a[e], O3, O2 + i2, p6, k0, full);
                         tma_load_4d(B, &M.b[e], k0, p4, p5, O1, full);
-                    } else {
-                        tma_load_4d(A, &M.a[e], k0, p4, O1, O2, full);
-                        tma_load_4d(B, &M.b[e], k0, O3, p6, p5, full);
                     }
+                } else {
+                    if (lane == 0) tma_load_4d(A, &M.a[e], k0, p4, O1, O2, full);
+                    if (lane == 1) tma_load_4d(B, &M.b[e], k0, O3, p6, p5, full);
                 }
             }
         }
@@ -683,6 +687,26 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
     // ==================================== consumers (warps 0..7)
     const int gq = lane >> 2, tq = lane & 3;
     const int tid = threadIdx.x;  // < 256
+    // t3 of the unit -> cube (cp.async, one group).  Full 16^3 cubes: thread t owns
+    // (q0, q1) = (t & 15, t >> 4) for every q2 — a constant stride per copy.
+    const int Q0 = P.qe[0], Q01 = P.qe[0] * P.qe[1];
+    auto seed = [&](const int* o, const int* len, int64_t pbase, double* cube) {
+        if (len[0] == BS && len[1] == BS && len[2] == BS) {
+            const int q0 = tid & 15, q1 = tid >> 4;
+            const double* src = P.t3 + pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)P.qe[1] * o[2]);
+            double* dst = cube + q0 + CST * q1;
+#pragma unroll
+            for (int q2 = 0; q2 < BS; ++q2) cp_async_8(dst + CST * CST * q2, src + (int64_t)Q01 * q2);
+        } else {
+            const int nvol = len[0] * len[1] * len[2];
+            for (int i = tid; i < nvol; i += 256) {
+                const int q0 = i % len[0], r = i / len[0];
+                const int q1 = r % len[1], q2 = r / len[1];
+                cp_async_8(cube + q0 + CST * (q1 + CST * q2),
+                           P.t3 + pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2)));
+            }
+        }
+    };
     int g = 0;
     for (int u = blockIdx.x; u < units; u += gridDim.x) {
         int o[3], len[3], qv[3];
@@ -690,15 +714,11 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
         const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
                               (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
         const int nvol = len[0] * len[1] * len[2];
-        for (int i = tid; i < nvol; i += 256) {
-            const int q0 = i % len[0], r = i / len[0];
-            const int q1 = r % len[1], q2 = r / len[1];
-            cp_async_8(acc_s + q0 + CST * (q1 + CST * q2),
-                       P.t3 + pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2)));
-        }
+        named_bar_sync(1, 256);  // the previous unit's store from the cube is complete
+        seed(o, len, pbase, acc_s);  // lands while the first stages compute
         cp_async_commit();
-        cp_async_wait_all();
-        named_bar_sync(1, 256);
+        bool seeded = false;
+
 
         double c[4][2][2];
 #pragma unroll
@@ -741,6 +761,11 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
             if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
             const bool last_chunk = (k0 + KC >= K);
             if (last_chunk && (e + 1 == P.nentry || P.ecls[e + 1] != P.ecls[e])) {
+                if (!seeded) {  // this unit's t3 seed must have landed for everyone
+                    cp_async_wait_n<0>();
+                    named_bar_sync(1, 256);
+                    seeded = true;
+                }
                 const int cl = P.ecls[e];
                 const int h1p = P.hpos[cl][0], h2p = P.hpos[cl][1], h3p = P.hpos[cl][2];
                 const int s1 = h1p == 0 ? 1 : (h1p == 1 ? CST : CST * CST);
@@ -769,15 +794,27 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
                 }
             }
         }
-        named_bar_sync(1, 256);
-        for (int i = tid; i < nvol; i += 256) {
-            const int q0 = i % len[0], r = i / len[0];
-            const int q1 = r % len[1], q2 = r / len[1];
-            P.t3[pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2))] =
-                acc_s[q0 + CST * (q1 + CST * q2)];
+        if (!seeded) {
+            cp_async_wait_n<0>();
+            seeded = true;
         }
-        named_bar_sync(1, 256);
+        named_bar_sync(1, 256);  // all flushes into this cube are done
+        if (len[0] == BS && len[1] == BS && len[2] == BS) {
+            const int q0 = tid & 15, q1 = tid >> 4;
+            double* dstg = P.t3 + pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)P.qe[1] * o[2]);
+            const double* srcs = acc_s + q0 + CST * q1;
+#pragma unroll
+            for (int q2 = 0; q2 < BS; ++q2) dstg[(int64_t)Q01 * q2] = srcs[CST * CST * q2];
+        } else {
+            for (int i = tid; i < nvol; i += 256) {
+                const int q0 = i % len[0], r = i / len[0];
+                const int q1 = r % len[1], q2 = r / len[1];
+                P.t3[pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2))] =
+                    acc_s[q0 + CST * (q1 + CST * q2)];
+            }
+        }
     }
+    cp_async_wait_all();
 }
 
 // ---- host: tensor maps (driver entry point, no -lcuda)

@@ -125,7 +125,7 @@ struct Line {
 // chains per thread.  All reads of a line precede the writes of that line and every
 // line is read by exactly one thread, so `out` may overwrite the line in place.
 template <int P1, int NA, int AXIS, int R, int NT, typename T, typename Out>
-__device__ __forceinline__ void apply_lines(const T* in, const T* __restrict__ opT, int nlines, Out out) {
+__device__ __forceinline__ void apply_lines(const T* in, const T* opT, int nlines, Out out) {
     using G = Geo<P1, NA, T>;
     using LN = Line<P1, NA, AXIS, T>;
     using P2 = typename Pair<T>::type;
@@ -174,13 +174,23 @@ __device__ __forceinline__ void apply_lines(const T* in, const T* __restrict__ o
 }
 
 // operator staging: opT[n][k] = M[k][n], M = Mat (TRANSPOSE = false) or Mat^T (true)
+// Every lane runs the same number of iterations and the warp reconverges afterwards:
+// with a divergent early exit, ptxas (CUDA 12.9, sm_100a) let the exited lanes of a warp
+// reload the uniform register holding the NEXT operator's pointer while the other lanes
+// were still loading this one (found by tests/test_parity_spectral at P1 = 13 with 96
+// threads).
 template <int P1, typename T, int NT, bool TRANSPOSE = false>
 __device__ __forceinline__ void load_op(T* __restrict__ op_s, const T* __restrict__ Mat) {
     constexpr int OS = (P1 + 1) & ~1;
-    for (int i = threadIdx.x; i < P1 * OS; i += NT) {
-        const int n = i / OS, k = i - (i / OS) * OS;
-        op_s[i] = (k < P1) ? (TRANSPOSE ? Mat[n * P1 + k] : Mat[k * P1 + n]) : T(0);
+#pragma unroll
+    for (int i0 = 0; i0 < P1 * OS; i0 += NT) {
+        const int i = i0 + (int)threadIdx.x;
+        if (i < P1 * OS) {
+            const int n = i / OS, k = i - (i / OS) * OS;
+            op_s[i] = (k < P1) ? (TRANSPOSE ? Mat[n * P1 + k] : Mat[k * P1 + n]) : T(0);
+        }
     }
+    __syncwarp();
 }
 
 template <int P1, typename T>
@@ -195,16 +205,25 @@ __host__ __device__ __forceinline__ int imin64(int64_t a, int64_t b) { return (i
 // small fixed table"): elements per CTA group E, threads NT, lines per thread R, number
 // of element buffers NBUF.  All stages run in place, so a kernel needs one buffer per
 // live field (+1 for the prefetch of the next group).
-template <int P1, int NA, typename T, int NBUF>
-struct Cfg {
-    using G = Geo<P1, NA, T>;
-#ifndef BC_SPEC_BUF_KB
-#define BC_SPEC_BUF_KB 36
-#endif
+// Measured on B200 (tools/sweep_spectral.py, profiles/sweep_spectral_r01.jsonl): 18 KiB groups
+// win at P1 >= 10 for every kernel; 36 KiB groups win for local_grad3 below that.
+enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
 #ifndef BC_SPEC_R
 #define BC_SPEC_R 2
 #endif
-    static constexpr int BUF_BYTES = BC_SPEC_BUF_KB * 1024;  // target bytes per element-group buffer
+template <int P1, int KIND>
+constexpr int spec_buf_kb() {
+#ifdef BC_SPEC_BUF_KB
+    return BC_SPEC_BUF_KB;
+#else
+    return (P1 >= 10) ? 18 : (KIND == K_LG3 ? 36 : 18);
+#endif
+}
+
+template <int P1, int NA, typename T, int NBUF, int KIND = K_SF3>
+struct Cfg {
+    using G = Geo<P1, NA, T>;
+    static constexpr int BUF_BYTES = spec_buf_kb<P1, KIND>() * 1024;  // target bytes per element-group buffer
     static constexpr int E0 = BUF_BYTES / (G::ES * (int)sizeof(T));
     static constexpr int E = E0 < 2 ? 1 : (E0 & ~1);  // even: groups of odd-P1 elements stay 16B-aligned
     static constexpr int R = BC_SPEC_R;
@@ -300,11 +319,11 @@ int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, 
 // ====================================================================== sumfact2d
 //   W[l][j] = sum_m A[j][m] U[l][m]  (rows, in place);  V[i][j] = sum_l B[i][l] W[l][j]
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, 1, double, 2>::NT)
+__global__ void __launch_bounds__(Cfg<P1, 1, double, 2, K_SF2>::NT)
 sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restrict__ B,
                  const double* __restrict__ U, double* __restrict__ V) {
     using T = double;
-    using CF = Cfg<P1, 1, T, 2>;
+    using CF = Cfg<P1, 1, T, 2, K_SF2>;
     using G = Geo<P1, 1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -326,7 +345,7 @@ sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restri
 
 template <int P1>
 int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* U, double* V, cudaStream_t s) {
-    using CF = Cfg<P1, 1, double, 2>;
+    using CF = Cfg<P1, 1, double, 2, K_SF2>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(sumfact2d_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
@@ -339,11 +358,11 @@ int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* 
 // us and ut are stored from registers (coalesced); ur is formed in place (its rows are
 // strided across threads) and copied out coalesced.
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, 2>::NT)
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 2, K_LG3>::NT)
 local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ U,
                    double* __restrict__ ur, double* __restrict__ us, double* __restrict__ ut) {
     using T = double;
-    using CF = Cfg<P1, P1, T, 2>;
+    using CF = Cfg<P1, P1, T, 2, K_LG3>;
     using G = Geo<P1, P1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -370,7 +389,7 @@ local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __rest
 template <int P1>
 int launch_local_grad3(int64_t N, const double* D, const double* U, double* ur, double* us, double* ut,
                        cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, 2>;
+    using CF = Cfg<P1, P1, double, 2, K_LG3>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(local_grad3_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
@@ -382,11 +401,11 @@ int launch_local_grad3(int64_t N, const double* D, const double* U, double* ur, 
 //   U = D^T along axis 2 of ur + D^T along axis 1 of us + D^T along axis 0 of ut,
 //   partial sums added in the order (r + s) + t.  Three field buffers, all in place.
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, 3>::NT)
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 3, K_LG3T>::NT)
 local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ ur,
                      const double* __restrict__ us, const double* __restrict__ ut, double* __restrict__ U) {
     using T = double;
-    using CF = Cfg<P1, P1, T, 3>;
+    using CF = Cfg<P1, P1, T, 3, K_LG3T>;
     using G = Geo<P1, P1, T>;
     constexpr int E = CF::E, NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -423,7 +442,7 @@ local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __re
 template <int P1>
 int launch_local_grad3_t(int64_t N, const double* D, const double* ur, const double* us, const double* ut,
                          double* U, cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, 3>;
+    using CF = Cfg<P1, P1, double, 3, K_LG3T>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(local_grad3_t_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
@@ -435,11 +454,11 @@ int launch_local_grad3_t(int64_t N, const double* D, const double* ur, const dou
 // (us, ut) from U into two buffers; ur in place over U; per-point geometric mixing in
 // place; then local_grad3_t in place as above.  Three field buffers.
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, 3>::NT)
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 3, K_AXE>::NT)
 ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ Uin,
             const double* __restrict__ Gm, double* __restrict__ Wout) {
     using T = double;
-    using CF = Cfg<P1, P1, T, 3>;
+    using CF = Cfg<P1, P1, T, 3, K_AXE>;
     using G = Geo<P1, P1, T>;
     constexpr int E = CF::E, NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -494,7 +513,7 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
 
 template <int P1>
 int launch_ax_e(int64_t N, const double* D, const double* U, const double* Gm, double* W, cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, 3>;
+    using CF = Cfg<P1, P1, double, 3, K_AXE>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(ax_e_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
