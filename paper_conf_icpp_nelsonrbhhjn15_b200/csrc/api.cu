@@ -1,6 +1,7 @@
 // libbarracuda C ABI (include/barracuda.h): argument validation and dispatch.
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <mutex>
 
 #include "common.cuh"
@@ -15,11 +16,24 @@ int run_local_grad3_t(int64_t, int, const double*, const double*, const double*,
 int run_ax_e(int64_t, int, const double*, const double*, const double*, double*, cudaStream_t);
 int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const double* const* opA,
               const double* const* opB, cudaStream_t s);
+int run_sumfact3d_mma(int64_t, int, const double*, const double*, const double*, const double*, double*, cudaStream_t);
+int run_sumfact2d_mma(int64_t, int, const double*, const double*, const double*, double*, cudaStream_t);
+int run_local_grad3_mma(int64_t, int, const double*, const double*, double*, double*, double*, cudaStream_t);
 int run_sumsq(int64_t n, const double* x, double* ws, cudaStream_t s);
 int run_energy(const int* ext7, const double* t3, const double* eh, const double* ep, double* ws, cudaStream_t s);
 template <typename T>
 int run_fill(int kind, uint64_t seed, uint64_t tid, uint64_t offset, int64_t n, double lo, double hi, T* out,
              cudaStream_t s);
+
+// Tensor-core (DMMA) spectral kernels are used where they cover p (spectral_mma.cu); the
+// environment variable BC_SPECTRAL_PATH=dfma forces the DFMA kernels (A/B measurements).
+static bool spectral_mma_enabled() {
+    static const bool on = [] {
+        const char* v = getenv("BC_SPECTRAL_PATH");
+        return !(v && v[0] == 'd');
+    }();
+    return on;
+}
 
 static thread_local int g_last_cuda_error = 0;
 static thread_local int64_t g_launches = 0;
@@ -148,6 +162,10 @@ int bc_sumfact3d(int64_t N, int p, const double* A, const double* B, const doubl
     const size_t nb = (size_t)N * (p + 1) * (p + 1) * (p + 1) * 8, ob = (size_t)(p + 1) * (p + 1) * 8;
     BC_REQUIRE(!overlap(V, nb, U, nb) && !overlap(V, nb, A, ob) && !overlap(V, nb, B, ob) && !overlap(V, nb, C, ob),
                BC_ERR_ALIAS);
+    if (spectral_mma_enabled()) {
+        const int st2 = run_sumfact3d_mma(N, p, A, B, C, U, V, as_stream(stream));
+        if (st2 != 1) return st2;  // 1: p not covered by the tensor-core kernels
+    }
     return run_sumfact3d(N, p, A, B, C, U, V, as_stream(stream));
 }
 
@@ -170,6 +188,10 @@ int bc_sumfact2d(int64_t N, int p, const double* A, const double* B, const doubl
     BC_REQUIRE(aligned(A, 16) && aligned(B, 16) && aligned(U, 16) && aligned(V, 16), BC_ERR_ALIGN);
     const size_t nb = (size_t)N * (p + 1) * (p + 1) * 8, ob = (size_t)(p + 1) * (p + 1) * 8;
     BC_REQUIRE(!overlap(V, nb, U, nb) && !overlap(V, nb, A, ob) && !overlap(V, nb, B, ob), BC_ERR_ALIAS);
+    if (spectral_mma_enabled()) {
+        const int st2 = run_sumfact2d_mma(N, p, A, B, U, V, as_stream(stream));
+        if (st2 != 1) return st2;  // 1: p not covered by the tensor-core kernels
+    }
     return run_sumfact2d(N, p, A, B, U, V, as_stream(stream));
 }
 
@@ -184,6 +206,10 @@ int bc_local_grad3(int64_t N, int p, const double* D, const double* U, double* u
     for (int i = 0; i < 3; ++i) {
         BC_REQUIRE(!overlap(outs[i], nb, U, nb) && !overlap(outs[i], nb, D, ob), BC_ERR_ALIAS);
         for (int j = i + 1; j < 3; ++j) BC_REQUIRE(!overlap(outs[i], nb, outs[j], nb), BC_ERR_ALIAS);
+    }
+    if (spectral_mma_enabled()) {
+        const int st2 = run_local_grad3_mma(N, p, D, U, ur, us, ut, as_stream(stream));
+        if (st2 != 1) return st2;  // 1: p not covered by the tensor-core kernels
     }
     return run_local_grad3(N, p, D, U, ur, us, ut, as_stream(stream));
 }

@@ -850,7 +850,7 @@ static bool encode_4d(CUtensorMap* m, const double* ptr, const int* dims, const 
     return r == CUDA_SUCCESS;
 }
 
-// returns -1 when the TMA path is unavailable (caller falls back)
+// returns 1 when the TMA path is unavailable (caller falls back)
 template <int FAM>
 static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
     TmaMaps M;
@@ -868,7 +868,7 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
             const int db[4] = {K, H3, P6, P5}, bb[4] = {TmaGeo::KC, 16, 1, 1};
             ok = encode_4d(&M.a[e], P.opA[e], da, ba, false) && encode_4d(&M.b[e], P.opB[e], db, bb, false);
         }
-        if (!ok) return -1;
+        if (!ok) return 1;
     }
     static int occ = 0;
     if (occ == 0) {
@@ -952,8 +952,8 @@ int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const
                         getenv("BC_NO_MMA") == nullptr;
     const bool tma_ok = mma_ok && getenv("BC_NO_TMA") == nullptr;
     if (tma_ok) {
-        const int st = (fam == FAM_D1) ? launch_ccsdt_tma<FAM_D1>(P, s) : (fam == FAM_D2 ? launch_ccsdt_tma<FAM_D2>(P, s) : -1);
-        if (st != -1) return st;
+        const int st = (fam == FAM_D1) ? launch_ccsdt_tma<FAM_D1>(P, s) : (fam == FAM_D2 ? launch_ccsdt_tma<FAM_D2>(P, s) : 1);
+        if (st != 1) return st;  // 1: tensor maps unavailable
     }
     if (mma_ok && fam == FAM_D1) return launch_ccsdt_mma<FAM_D1>(P, s);
     if (mma_ok && fam == FAM_D2) return launch_ccsdt_mma<FAM_D2>(P, s);

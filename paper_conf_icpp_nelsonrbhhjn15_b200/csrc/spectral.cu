@@ -247,27 +247,45 @@ int grid_for(KernelT kernel, int nt, size_t smem, int64_t ngroups, int* occ_cach
     return imin64(ngroups, cap);
 }
 
-// Group loop with a one-group-ahead cp.async prefetch of the single input field:
-//   body(in, e0, ne) processes group starting at element e0 held in smem `in`.
+// Group loop over the single input field.  PREFETCH: one-group-ahead cp.async prefetch
+// into a second buffer; otherwise load -> wait -> compute, with latency hidden by the
+// other CTAs on the SM (twice as many fit).
+#ifndef BC_SPEC_PREFETCH
+#define BC_SPEC_PREFETCH 1
+#endif
+constexpr int SPEC_NBUF1 = BC_SPEC_PREFETCH ? 2 : 1;  // buffers for single-field kernels
+
 template <int P1, int NA, typename T, int NT, int E, int BUF, typename Body>
 __device__ __forceinline__ void group_loop_prefetch(int64_t N, const T* __restrict__ src, T* buf0, Body body) {
     using G = Geo<P1, NA, T>;
     const int64_t ngroups = (N + E - 1) / E;
-    int64_t g = blockIdx.x;
-    if (g < ngroups) load_group_async<P1, NA, T, NT>(buf0, src + g * E * G::NPTS, imin64(E, N - g * E));
-    cp_async_commit();
-    int cur = 0;
-    for (; g < ngroups; g += gridDim.x) {
-        const int64_t e0 = g * E;
-        cp_async_wait_all();
-        __syncthreads();  // group g landed; everyone is done with the other buffer
-        T* in = buf0 + cur * BUF;
-        const int64_t gn = g + gridDim.x;
-        if (gn < ngroups)
-            load_group_async<P1, NA, T, NT>(buf0 + (cur ^ 1) * BUF, src + gn * E * G::NPTS, imin64(E, N - gn * E));
+    if constexpr (BC_SPEC_PREFETCH) {
+        int64_t g = blockIdx.x;
+        if (g < ngroups) load_group_async<P1, NA, T, NT>(buf0, src + g * E * G::NPTS, imin64(E, N - g * E));
         cp_async_commit();
-        body(in, e0, imin64(E, N - e0));
-        cur ^= 1;
+        int cur = 0;
+        for (; g < ngroups; g += gridDim.x) {
+            const int64_t e0 = g * E;
+            cp_async_wait_all();
+            __syncthreads();  // group g landed; everyone is done with the other buffer
+            T* in = buf0 + cur * BUF;
+            const int64_t gn = g + gridDim.x;
+            if (gn < ngroups)
+                load_group_async<P1, NA, T, NT>(buf0 + (cur ^ 1) * BUF, src + gn * E * G::NPTS, imin64(E, N - gn * E));
+            cp_async_commit();
+            body(in, e0, imin64(E, N - e0));
+            cur ^= 1;
+        }
+    } else {
+        for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
+            const int64_t e0 = g * E;
+            __syncthreads();  // everyone is done with the buffer
+            load_group_async<P1, NA, T, NT>(buf0, src + e0 * G::NPTS, imin64(E, N - e0));
+            cp_async_commit();
+            cp_async_wait_all();
+            __syncthreads();
+            body(buf0, e0, imin64(E, N - e0));
+        }
     }
 }
 
@@ -278,10 +296,10 @@ __device__ __forceinline__ void group_loop_prefetch(int64_t N, const T* __restri
 // S1 and S2 run in place in the group buffer; S3 stores V straight from registers
 // (consecutive threads own consecutive (j,k): coalesced).
 template <int P1, typename T>
-__global__ void __launch_bounds__(Cfg<P1, P1, T, 2>::NT)
+__global__ void __launch_bounds__(Cfg<P1, P1, T, SPEC_NBUF1>::NT)
 sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, const T* __restrict__ C,
                  const T* __restrict__ U, T* __restrict__ V) {
-    using CF = Cfg<P1, P1, T, 2>;
+    using CF = Cfg<P1, P1, T, SPEC_NBUF1>;
     using G = Geo<P1, P1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -307,7 +325,7 @@ sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, co
 
 template <int P1, typename T>
 int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, cudaStream_t s) {
-    using CF = Cfg<P1, P1, T, 2>;
+    using CF = Cfg<P1, P1, T, SPEC_NBUF1>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const size_t smem = CF::SMEM + op_elems<P1, T>() * sizeof(T);
@@ -319,11 +337,11 @@ int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, 
 // ====================================================================== sumfact2d
 //   W[l][j] = sum_m A[j][m] U[l][m]  (rows, in place);  V[i][j] = sum_l B[i][l] W[l][j]
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, 1, double, 2, K_SF2>::NT)
+__global__ void __launch_bounds__(Cfg<P1, 1, double, SPEC_NBUF1, K_SF2>::NT)
 sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restrict__ B,
                  const double* __restrict__ U, double* __restrict__ V) {
     using T = double;
-    using CF = Cfg<P1, 1, T, 2, K_SF2>;
+    using CF = Cfg<P1, 1, T, SPEC_NBUF1, K_SF2>;
     using G = Geo<P1, 1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -345,7 +363,7 @@ sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restri
 
 template <int P1>
 int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* U, double* V, cudaStream_t s) {
-    using CF = Cfg<P1, 1, double, 2, K_SF2>;
+    using CF = Cfg<P1, 1, double, SPEC_NBUF1, K_SF2>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(sumfact2d_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
@@ -358,11 +376,11 @@ int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* 
 // us and ut are stored from registers (coalesced); ur is formed in place (its rows are
 // strided across threads) and copied out coalesced.
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, 2, K_LG3>::NT)
+__global__ void __launch_bounds__(Cfg<P1, P1, double, SPEC_NBUF1, K_LG3>::NT)
 local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ U,
                    double* __restrict__ ur, double* __restrict__ us, double* __restrict__ ut) {
     using T = double;
-    using CF = Cfg<P1, P1, T, 2, K_LG3>;
+    using CF = Cfg<P1, P1, T, SPEC_NBUF1, K_LG3>;
     using G = Geo<P1, P1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -389,7 +407,7 @@ local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __rest
 template <int P1>
 int launch_local_grad3(int64_t N, const double* D, const double* U, double* ur, double* us, double* ut,
                        cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, 2, K_LG3>;
+    using CF = Cfg<P1, P1, double, SPEC_NBUF1, K_LG3>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(local_grad3_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);

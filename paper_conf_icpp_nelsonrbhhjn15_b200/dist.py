@@ -22,13 +22,17 @@ class Rank:
 
 def init(backend: str | None = None) -> Rank:
     """Read RANK / WORLD_SIZE / LOCAL_RANK (torchrun); init the process group if world > 1.
-    backend defaults to nccl when CUDA is available, else gloo."""
+    backend defaults to nccl when CUDA is available, else gloo (BC_DIST_BACKEND overrides;
+    with more ranks than GPUs — a test configuration — ranks share GPUs modulo the count
+    and must use gloo, since NCCL needs one GPU per rank)."""
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    backend = backend or os.environ.get("BC_DIST_BACKEND")
     if torch.cuda.is_available():
-        torch.cuda.set_device(local)
-        device = torch.device("cuda", local)
+        dev_index = local % torch.cuda.device_count()
+        torch.cuda.set_device(dev_index)
+        device = torch.device("cuda", dev_index)
     else:
         device = torch.device("cpu")
     if world > 1 and not dist.is_initialized():
@@ -61,19 +65,33 @@ def owner(unit: int, n: int, world: int) -> int:
 
 def barrier() -> None:
     if dist.is_initialized():
-        dist.barrier()
+        if dist.get_backend() == "nccl":
+            dist.barrier(device_ids=[torch.cuda.current_device()])
+        else:
+            dist.barrier()
+
+
+def _coll_device(device: torch.device) -> torch.device:
+    # gloo reduces host tensors; NCCL device tensors
+    return device if dist.get_backend() == "nccl" else torch.device("cpu")
 
 
 def all_reduce_sum_(t: torch.Tensor) -> torch.Tensor:
     """In-place SUM of a (small) check tensor over ranks; identity when world == 1."""
     if dist.is_initialized() and dist.get_world_size() > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        cd = _coll_device(t.device)
+        if cd == t.device:
+            dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        else:
+            h = t.to(cd)
+            dist.all_reduce(h, op=dist.ReduceOp.SUM)
+            t.copy_(h)
     return t
 
 
 def max_over_ranks(x: float, device: torch.device) -> float:
     if dist.is_initialized() and dist.get_world_size() > 1:
-        t = torch.tensor([x], dtype=torch.float64, device=device)
+        t = torch.tensor([x], dtype=torch.float64, device=_coll_device(device))
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
     return x
