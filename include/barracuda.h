@@ -64,6 +64,11 @@ typedef enum {
  * paper(A,B,C,U) = bc_sumfact3d(A^T, B^T, C^T, reverse_axes(U)). */
 int bc_sumfact3d(int64_t N, int p, const double* A, const double* B, const double* C,
                  const double* U, double* V, void* stream);
+/* Same, plus the check scalar ws[0] = sum over all V of V^2 (R18), accumulated in the
+ * kernel's store epilogue instead of re-reading V (ws: device workspace of
+ * >= BC_CHECK_WS_DOUBLES doubles, deterministic fixed-order reduction). */
+int bc_sumfact3d_check(int64_t N, int p, const double* A, const double* B, const double* C,
+                       const double* U, double* V, double* ws, void* stream);
 /* Same in fp32 (R16). */
 int bc_sumfact3d_f32(int64_t N, int p, const float* A, const float* B, const float* C,
                      const float* U, float* V, void* stream);

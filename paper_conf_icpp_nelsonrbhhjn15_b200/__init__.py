@@ -72,12 +72,20 @@ def _field(U: torch.Tensor, P1: int, ndim: int, name: str) -> int:
 
 # ----------------------------------------------------------------------------- spectral
 
-def sumfact3d(A, B, C, U, out: Optional[torch.Tensor] = None) -> torch.Tensor:
-    """V[e][i][j][k] = sum_lmn A[k][n] B[j][m] C[i][l] U[e][l][m][n]  (fp64 or fp32)."""
+def sumfact3d(A, B, C, U, out: Optional[torch.Tensor] = None, check_ws: Optional[torch.Tensor] = None) -> torch.Tensor:
+    """V[e][i][j][k] = sum_lmn A[k][n] B[j][m] C[i][l] U[e][l][m][n]  (fp64 or fp32).
+    check_ws (fp64, >= 1024 doubles): also leave sum(V^2) in check_ws[0] (fused, fp64 only)."""
     p = _p_of(A, "A")
     N = _field(U, p + 1, 3, "U")
     V = torch.empty_like(U) if out is None else out
     dt = U.dtype
+    if check_ws is not None:
+        f = torch.float64
+        if check_ws.numel() < BC_CHECK_WS_DOUBLES:
+            raise ValueError("check_ws needs >= 1024 doubles")
+        _check(lib.bc_sumfact3d_check(N, p, _dev(A, f, "A"), _dev(B, f, "B"), _dev(C, f, "C"), _dev(U, f, "U"),
+                                      _dev(V, f, "out"), _dev(check_ws, f, "check_ws"), _stream(U)), "bc_sumfact3d_check")
+        return V
     fn = {torch.float64: lib.bc_sumfact3d, torch.float32: lib.bc_sumfact3d_f32}.get(dt)
     if fn is None:
         raise TypeError("sumfact3d supports float64 and float32")

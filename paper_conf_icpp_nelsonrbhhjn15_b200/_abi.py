@@ -29,6 +29,7 @@ PtrArray9 = _vp * 9
 
 _SIGS = {
     "bc_sumfact3d": [_i64, _i32, _vp, _vp, _vp, _vp, _vp, _vp],
+    "bc_sumfact3d_check": [_i64, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp],
     "bc_sumfact3d_f32": [_i64, _i32, _vp, _vp, _vp, _vp, _vp, _vp],
     "bc_sumfact2d": [_i64, _i32, _vp, _vp, _vp, _vp, _vp],
     "bc_local_grad3": [_i64, _i32, _vp, _vp, _vp, _vp, _vp, _vp],

@@ -8,7 +8,8 @@
 
 namespace bc {
 
-int run_sumfact3d(int64_t, int, const double*, const double*, const double*, const double*, double*, cudaStream_t);
+int run_sumfact3d(int64_t, int, const double*, const double*, const double*, const double*, double*, double*,
+                  cudaStream_t);
 int run_sumfact3d_f32(int64_t, int, const float*, const float*, const float*, const float*, float*, cudaStream_t);
 int run_sumfact2d(int64_t, int, const double*, const double*, const double*, double*, cudaStream_t);
 int run_local_grad3(int64_t, int, const double*, const double*, double*, double*, double*, cudaStream_t);
@@ -16,7 +17,8 @@ int run_local_grad3_t(int64_t, int, const double*, const double*, const double*,
 int run_ax_e(int64_t, int, const double*, const double*, const double*, double*, cudaStream_t);
 int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const double* const* opA,
               const double* const* opB, cudaStream_t s);
-int run_sumfact3d_mma(int64_t, int, const double*, const double*, const double*, const double*, double*, cudaStream_t);
+int run_sumfact3d_mma(int64_t, int, const double*, const double*, const double*, const double*, double*, double*,
+                      cudaStream_t);
 int run_sumfact2d_mma(int64_t, int, const double*, const double*, const double*, double*, cudaStream_t);
 int run_local_grad3_mma(int64_t, int, const double*, const double*, double*, double*, double*, cudaStream_t);
 int run_sumsq(int64_t n, const double* x, double* ws, cudaStream_t s);
@@ -147,6 +149,29 @@ static int ccsdt_fused(int fam, const bc_tile_dims* d, double* t3, const double*
     return BC_OK;
 }
 
+static int sumfact3d_impl(int64_t N, int p, const double* A, const double* B, const double* C, const double* U,
+                          double* V, double* ws, void* stream) {
+    int st = check_spectral(N, p);
+    if (st) return st;
+    BC_REQUIRE(ws == nullptr || aligned(ws, 8), BC_ERR_ALIGN);
+    if (N == 0) {
+        if (ws) return run_sumsq(0, V, ws, as_stream(stream));  // ws[0] = 0
+        return BC_OK;
+    }
+    BC_REQUIRE(A && B && C && U && V, BC_ERR_ARG);
+    BC_REQUIRE(aligned(A, 16) && aligned(B, 16) && aligned(C, 16) && aligned(U, 16) && aligned(V, 16), BC_ERR_ALIGN);
+    const size_t nb = (size_t)N * (p + 1) * (p + 1) * (p + 1) * 8, ob = (size_t)(p + 1) * (p + 1) * 8;
+    BC_REQUIRE(!overlap(V, nb, U, nb) && !overlap(V, nb, A, ob) && !overlap(V, nb, B, ob) && !overlap(V, nb, C, ob),
+               BC_ERR_ALIAS);
+    BC_REQUIRE(!ws || (!overlap(ws, BC_CHECK_WS_DOUBLES * 8, V, nb) && !overlap(ws, BC_CHECK_WS_DOUBLES * 8, U, nb)),
+               BC_ERR_ALIAS);
+    if (spectral_mma_enabled()) {
+        const int st2 = run_sumfact3d_mma(N, p, A, B, C, U, V, ws, as_stream(stream));
+        if (st2 != 1) return st2;  // 1: p not covered by the tensor-core kernels
+    }
+    return run_sumfact3d(N, p, A, B, C, U, V, ws, as_stream(stream));
+}
+
 }  // namespace bc
 
 using namespace bc;
@@ -155,18 +180,13 @@ extern "C" {
 
 int bc_sumfact3d(int64_t N, int p, const double* A, const double* B, const double* C, const double* U,
                  double* V, void* stream) {
-    int st = check_spectral(N, p);
-    if (st || N == 0) return st;
-    BC_REQUIRE(A && B && C && U && V, BC_ERR_ARG);
-    BC_REQUIRE(aligned(A, 16) && aligned(B, 16) && aligned(C, 16) && aligned(U, 16) && aligned(V, 16), BC_ERR_ALIGN);
-    const size_t nb = (size_t)N * (p + 1) * (p + 1) * (p + 1) * 8, ob = (size_t)(p + 1) * (p + 1) * 8;
-    BC_REQUIRE(!overlap(V, nb, U, nb) && !overlap(V, nb, A, ob) && !overlap(V, nb, B, ob) && !overlap(V, nb, C, ob),
-               BC_ERR_ALIAS);
-    if (spectral_mma_enabled()) {
-        const int st2 = run_sumfact3d_mma(N, p, A, B, C, U, V, as_stream(stream));
-        if (st2 != 1) return st2;  // 1: p not covered by the tensor-core kernels
-    }
-    return run_sumfact3d(N, p, A, B, C, U, V, as_stream(stream));
+    return sumfact3d_impl(N, p, A, B, C, U, V, nullptr, stream);
+}
+
+int bc_sumfact3d_check(int64_t N, int p, const double* A, const double* B, const double* C, const double* U,
+                       double* V, double* ws, void* stream) {
+    BC_REQUIRE(ws != nullptr, BC_ERR_ARG);
+    return sumfact3d_impl(N, p, A, B, C, U, V, ws, stream);
 }
 
 int bc_sumfact3d_f32(int64_t N, int p, const float* A, const float* B, const float* C, const float* U, float* V,

@@ -96,6 +96,11 @@ static int red_blocks(int64_t n) {
     return b < 1 ? 1 : (int)b;
 }
 
+int run_check_finalize(int nparts, double* ws, cudaStream_t s) {
+    finalize<<<1, RED_NT, 0, s>>>(nparts, ws + 8, ws);
+    return launch_status();
+}
+
 int run_sumsq(int64_t n, const double* x, double* ws, cudaStream_t s) {
     const int nb = red_blocks(n);
     sumsq_partial<<<nb, RED_NT, 0, s>>>(n, x, ws + 8);

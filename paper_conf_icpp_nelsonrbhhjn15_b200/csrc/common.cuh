@@ -24,6 +24,27 @@ inline int launch_status() {
 
 inline cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
 
+// ---------------------------------------------------------------- fused check partials
+// Kernels that fuse a check scalar write one fp64 partial per CTA to ws[8 + blockIdx.x]
+// (at most CHECK_MAX_PARTIALS CTAs); run_check_finalize sums them in fixed order to ws[0].
+constexpr int CHECK_MAX_PARTIALS = BC_CHECK_WS_DOUBLES - 8;
+int run_check_finalize(int nparts, double* ws, cudaStream_t s);
+
+// block-wide sum of v; thread 0 writes part[blockIdx.x]  (all threads must call)
+__device__ __forceinline__ void block_partial(double v, double* part) {
+    __shared__ double red[32];
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+    __syncthreads();
+    if (l == 0) red[w] = v;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double s = 0.0;
+        for (int i = 0; i < (int)((blockDim.x + 31) >> 5); ++i) s += red[i];
+        part[blockIdx.x] = s;
+    }
+}
+
 // ---------------------------------------------------------------- cp.async (LDGSTS)
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));

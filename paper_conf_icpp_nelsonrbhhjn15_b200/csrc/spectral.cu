@@ -294,11 +294,13 @@ __device__ __forceinline__ void group_loop_prefetch(int64_t N, const T* __restri
 //   S2 W2[l][j][k] = sum_m B[j][m] W1[l][m][k]    (axis 1, P:441 / P:214)
 //   S3 V [i][j][k] = sum_l C[i][l] W2[l][j][k]    (axis 0, P:442 / P:215; Fig. 2(d))
 // S1 and S2 run in place in the group buffer; S3 stores V straight from registers
-// (consecutive threads own consecutive (j,k): coalesced).
+// (consecutive threads own consecutive (j,k): coalesced).  With ws != nullptr the check
+// scalar sum V^2 (R18) is accumulated in the store epilogue: one partial per
+// CTA in ws[8 + blockIdx.x], reduced in fixed order by check_finalize.
 template <int P1, typename T>
 __global__ void __launch_bounds__(Cfg<P1, P1, T, SPEC_NBUF1>::NT)
 sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, const T* __restrict__ C,
-                 const T* __restrict__ U, T* __restrict__ V) {
+                 const T* __restrict__ U, T* __restrict__ V, double* __restrict__ ws) {
     using CF = Cfg<P1, P1, T, SPEC_NBUF1>;
     using G = Geo<P1, P1, T>;
     constexpr int NT = CF::NT, R = CF::R;
@@ -310,6 +312,7 @@ sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, co
     load_op<P1, T, NT>(opA, A);
     load_op<P1, T, NT>(opB, B);
     load_op<P1, T, NT>(opC, C);
+    double sq = 0.0;
     group_loop_prefetch<P1, P1, T, NT, CF::E, CF::BUF>(N, U, buf, [&](T* in, int64_t e0, int ne) {
         const int nlines = ne * P1 * P1;
         apply_lines<P1, P1, 2, R, NT>(in, opA, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
@@ -319,19 +322,24 @@ sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, co
         T* Vg = V + e0 * G::NPTS;
         apply_lines<P1, P1, 0, R, NT>(in, opC, nlines, [&](int L, int, int k, T v) {
             st_cs(Vg + Line<P1, P1, 0, T>::gofs(L, k), v);
+            sq = fma((double)v, (double)v, sq);
         });
     });
+    if (ws != nullptr) block_partial(sq, ws + 8);
 }
 
 template <int P1, typename T>
-int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, cudaStream_t s) {
+int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, double* ws, cudaStream_t s) {
     using CF = Cfg<P1, P1, T, SPEC_NBUF1>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const size_t smem = CF::SMEM + op_elems<P1, T>() * sizeof(T);
-    const int grid = grid_for(sumfact3d_kernel<P1, T>, CF::NT, smem, ngroups, &occ);
-    sumfact3d_kernel<P1, T><<<grid, CF::NT, smem, s>>>(N, A, B, C, U, V);
-    return launch_status();
+    int grid = grid_for(sumfact3d_kernel<P1, T>, CF::NT, smem, ngroups, &occ);
+    if (ws && grid > CHECK_MAX_PARTIALS) grid = CHECK_MAX_PARTIALS;
+    sumfact3d_kernel<P1, T><<<grid, CF::NT, smem, s>>>(N, A, B, C, U, V, ws);
+    const int st = launch_status();
+    if (st || !ws) return st;
+    return run_check_finalize(grid, ws, s);
 }
 
 // ====================================================================== sumfact2d
@@ -561,14 +569,14 @@ int launch_ax_e(int64_t N, const double* D, const double* U, const double* Gm, d
     }
 
 int run_sumfact3d(int64_t N, int p, const double* A, const double* B, const double* C, const double* U,
-                  double* V, cudaStream_t s) {
-#define CALL(P) launch_sumfact3d<P, double>(N, A, B, C, U, V, s)
+                  double* V, double* ws, cudaStream_t s) {
+#define CALL(P) launch_sumfact3d<P, double>(N, A, B, C, U, V, ws, s)
     BC_P1_SWITCH(p + 1, CALL)
 #undef CALL
 }
 int run_sumfact3d_f32(int64_t N, int p, const float* A, const float* B, const float* C, const float* U,
                       float* V, cudaStream_t s) {
-#define CALL(P) launch_sumfact3d<P, float>(N, A, B, C, U, V, s)
+#define CALL(P) launch_sumfact3d<P, float>(N, A, B, C, U, V, nullptr, s)
     BC_P1_SWITCH(p + 1, CALL)
 #undef CALL
 }

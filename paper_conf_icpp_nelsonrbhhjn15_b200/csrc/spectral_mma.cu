@@ -185,11 +185,13 @@ __global__ void __launch_bounds__(MCfg<P1, P1>::NT) sumfact3d_mma_kernel(int64_t
                                                                        const double* __restrict__ B,
                                                                        const double* __restrict__ C,
                                                                        const double* __restrict__ U,
-                                                                       double* __restrict__ V) {
+                                                                       double* __restrict__ V,
+                                                                       double* __restrict__ ws) {
     using G = MG<P1, P1>;
     constexpr int NW = MCfg<P1, P1>::NW;
     extern __shared__ __align__(16) double smd[];
     double aA[G::MF][G::KS], aB[G::MF][G::KS], aC[G::MF][G::KS];
+    double sq = 0.0;
     load_afrag<P1>(aA, A);
     load_afrag<P1>(aB, B);
     load_afrag<P1>(aC, C);
@@ -205,8 +207,10 @@ __global__ void __launch_bounds__(MCfg<P1, P1>::NT) sumfact3d_mma_kernel(int64_t
         double* Vg = V + e0 * G::NPTS;
         mma_stage<P1, P1, 2, NW>(in, aA, ne, [&](int e, int l, int k, double v) {
             st_cs(Vg + e * G::NPTS + ML<P1, P1, 2>::gofs(l, k), v);
+            sq = fma(v, v, sq);
         });
     });
+    if (ws != nullptr) block_partial(sq, ws + 8);
 }
 
 // ------------------------------------------------------------------ sumfact2d
@@ -277,12 +281,15 @@ static int mma_grid(K kernel, size_t smem, int nt, int64_t ngroups, int* occ) {
 
 template <int P1>
 static int launch_sf3d_mma(int64_t N, const double* A, const double* B, const double* C, const double* U, double* V,
-                           cudaStream_t s) {
+                           double* ws, cudaStream_t s) {
     using CF = MCfg<P1, P1>;
     static int occ = 0;
-    const int grid = mma_grid(sumfact3d_mma_kernel<P1>, CF::SMEM, CF::NT, (N + CF::E - 1) / CF::E, &occ);
-    sumfact3d_mma_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, A, B, C, U, V);
-    return launch_status();
+    int grid = mma_grid(sumfact3d_mma_kernel<P1>, CF::SMEM, CF::NT, (N + CF::E - 1) / CF::E, &occ);
+    if (ws && grid > CHECK_MAX_PARTIALS) grid = CHECK_MAX_PARTIALS;
+    sumfact3d_mma_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, A, B, C, U, V, ws);
+    const int st = launch_status();
+    if (st || !ws) return st;
+    return run_check_finalize(grid, ws, s);
 }
 template <int P1>
 static int launch_sf2d_mma(int64_t N, const double* A, const double* B, const double* U, double* V, cudaStream_t s) {
@@ -316,8 +323,8 @@ static int launch_lg3_mma(int64_t N, const double* D, const double* U, double* u
     }
 
 int run_sumfact3d_mma(int64_t N, int p, const double* A, const double* B, const double* C, const double* U, double* V,
-                      cudaStream_t s) {
-#define CALL(P) launch_sf3d_mma<P>(N, A, B, C, U, V, s)
+                      double* ws, cudaStream_t s) {
+#define CALL(P) launch_sf3d_mma<P>(N, A, B, C, U, V, ws, s)
     BC_MMA_SWITCH(p + 1, CALL)
 #undef CALL
 }

@@ -21,7 +21,7 @@ import torch
 
 import synthetic as syn
 
-from . import ccsdt_fused, check_energy, check_sumsq, fill, local_grad3, sumfact2d, sumfact3d
+from . import ccsdt_fused, check_energy, fill, local_grad3, sumfact2d, sumfact3d
 from . import dist as bdist
 
 
@@ -45,12 +45,11 @@ def flops_bytes(cfg: StepConfig) -> dict:
     nop = t ** 4
     out = {
         "local_grad3": (6.0 * P1 ** 4 * N, 32.0 * P1 ** 3 * N),
-        "sumfact3d": (6.0 * P1 ** 4 * N, 16.0 * P1 ** 3 * N),
+        "sumfact3d": (6.0 * P1 ** 4 * N + 2.0 * P1 ** 3 * N, 16.0 * P1 ** 3 * N),  # + fused sum V^2
         "sumfact2d": (4.0 * P1 ** 3 * (N * P1), 16.0 * P1 ** 2 * (N * P1)),
     }
     for fam in cfg.families:
         out[f"ccsdt_{fam}_fused"] = (9 * 2.0 * n3 * t, 16.0 * n3 + 9 * 8.0 * 2 * nop)
-    out["check_sumsq"] = (2.0 * P1 ** 3 * N, 8.0 * P1 ** 3 * N)
     out["check_energy"] = (9.0 * n3, 8.0 * n3)
     return out
 
@@ -114,7 +113,7 @@ class Step:
         tick = timer or (lambda name: None)
         local_grad3(self.D, self.U, out=(self.ur, self.us, self.ut))
         tick("local_grad3")
-        sumfact3d(self.A, self.B, self.C, self.U, out=self.V)
+        sumfact3d(self.A, self.B, self.C, self.U, out=self.V, check_ws=self.ws[0])  # + fused sum V^2
         tick("sumfact3d")
         sumfact2d(self.A, self.B, self.U2, out=self.V2)
         tick("sumfact2d")
@@ -122,8 +121,6 @@ class Step:
             for b in range(c.blocks):
                 ccsdt_fused(fam, self.ext, self.t3[b], self.t2[(fam, b)], self.v2[(fam, b)])
             tick(f"ccsdt_{fam}_fused")
-        check_sumsq(self.V, self.ws[0])
-        tick("check_sumsq")
         for b in range(c.blocks):
             check_energy(self.ext, self.t3[b], self.eps_h, self.eps_p, self.ws[1 + b])
         tick("check_energy")
@@ -136,7 +133,7 @@ class Step:
         c = self.cfg
         return {"local_grad3": 1, "sumfact3d": 1, "sumfact2d": 1,
                 **{f"ccsdt_{f}_fused": c.blocks for f in c.families},
-                "check_sumsq": 2, "check_energy": 2 * c.blocks}
+                "check_energy": 2 * c.blocks}
 
     def flops_per_step(self) -> float:
         c = self.cfg

@@ -156,3 +156,16 @@ def test_errors_raise(bc):
     U = torch.zeros(3, 5, 5, 5, dtype=torch.float64, device="cuda")
     with pytest.raises(bc.BarracudaError, match="ALIAS"):
         bc.sumfact3d(A, A, A, U, out=U)
+
+
+@pytest.mark.parametrize("P1", [2, 5, 13, 16])
+def test_sumfact3d_fused_check_scalar(bc, P1):
+    """bc_sumfact3d_check: V as bc_sumfact3d, plus ws[0] = sum V^2 from the store epilogue."""
+    A, B, C = (syn.tensor(t, (P1, P1)) for t in (2, 3, 4))
+    U = syn.tensor(1, (301, P1, P1, P1))
+    ws = torch.full((1024,), float("nan"), dtype=torch.float64, device="cuda")
+    V = bc.sumfact3d(to_dev(A), to_dev(B), to_dev(C), to_dev(U), check_ws=ws)
+    Vr = oracle.sumfact3d(A, B, C, U)
+    assert_abs_close(to_host(V), Vr, oracle.sumfact3d(abs(A), abs(B), abs(C), abs(U)), 1e-12, "V")
+    ref = oracle.sumsq(Vr)
+    assert abs(ws[0].item() - ref) <= 1e-12 * ref
