@@ -205,28 +205,30 @@ __host__ __device__ __forceinline__ int imin64(int64_t a, int64_t b) { return (i
 // small fixed table"): elements per CTA group E, threads NT, lines per thread R, number
 // of element buffers NBUF.  All stages run in place, so a kernel needs one buffer per
 // live field (+1 for the prefetch of the next group).
-// Measured on B200 (tools/sweep_spectral.py, profiles/sweep_spectral_r01.jsonl): 18 KiB groups
-// win at P1 >= 10 for every kernel; 36 KiB groups win for local_grad3 below that.
+// Variant table, measured on B200 with tools/sweep_spectral.py (profiles/sweep_spectral_r01.md):
+//   P1 >= 10: sumfact3d / local_grad3: R = 4 lines per thread, 54 KiB element groups, no
+//             in-CTA prefetch (occupancy hides the loads); sumfact2d: R = 3, 18 KiB groups
+//             with prefetch; local_grad3_t / ax_e: R = 2, 18 KiB.
+//   P1 <  10: R = 2, 18 KiB groups with prefetch (36 KiB for local_grad3).
 enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
-#ifndef BC_SPEC_R
-#define BC_SPEC_R 2
-#endif
 template <int P1, int KIND>
-constexpr int spec_buf_kb() {
-#ifdef BC_SPEC_BUF_KB
-    return BC_SPEC_BUF_KB;
-#else
-    return (P1 >= 10) ? 18 : (KIND == K_LG3 ? 36 : 18);
-#endif
-}
+struct SpecTable {
+    static constexpr bool BIG = P1 >= 10;
+    static constexpr int R = BIG ? (KIND == K_SF3 || KIND == K_LG3 ? 4 : (KIND == K_SF2 ? 3 : 2)) : 2;
+    static constexpr int BUF_KB = BIG ? (KIND == K_SF3 || KIND == K_LG3 ? 54 : 18) : (KIND == K_LG3 ? 36 : 18);
+    static constexpr bool PREFETCH = !(BIG && (KIND == K_SF3 || KIND == K_LG3));
+};
 
-template <int P1, int NA, typename T, int NBUF, int KIND = K_SF3>
+template <int P1, int NA, typename T, int NBUF_FIELDS, int KIND = K_SF3>
 struct Cfg {
     using G = Geo<P1, NA, T>;
-    static constexpr int BUF_BYTES = spec_buf_kb<P1, KIND>() * 1024;  // target bytes per element-group buffer
+    using TB = SpecTable<P1, KIND>;
+    static constexpr bool PREFETCH = TB::PREFETCH && NBUF_FIELDS == 1;  // single-field kernels only
+    static constexpr int NBUF = NBUF_FIELDS + (PREFETCH ? 1 : 0);
+    static constexpr int BUF_BYTES = TB::BUF_KB * 1024;  // target bytes per element-group buffer
     static constexpr int E0 = BUF_BYTES / (G::ES * (int)sizeof(T));
     static constexpr int E = E0 < 2 ? 1 : (E0 & ~1);  // even: groups of odd-P1 elements stay 16B-aligned
-    static constexpr int R = BC_SPEC_R;
+    static constexpr int R = TB::R;
     static constexpr int LINES = E * NA * P1;  // lines per axis per group (E * NPTS / P1)
     static constexpr int NT0 = ((LINES + R - 1) / R + 31) / 32 * 32;
     static constexpr int NT = NT0 < 64 ? 64 : (NT0 > 512 ? 512 : NT0);
@@ -248,18 +250,13 @@ int grid_for(KernelT kernel, int nt, size_t smem, int64_t ngroups, int* occ_cach
 }
 
 // Group loop over the single input field.  PREFETCH: one-group-ahead cp.async prefetch
-// into a second buffer; otherwise load -> wait -> compute, with latency hidden by the
-// other CTAs on the SM (twice as many fit).
-#ifndef BC_SPEC_PREFETCH
-#define BC_SPEC_PREFETCH 1
-#endif
-constexpr int SPEC_NBUF1 = BC_SPEC_PREFETCH ? 2 : 1;  // buffers for single-field kernels
-
-template <int P1, int NA, typename T, int NT, int E, int BUF, typename Body>
-__device__ __forceinline__ void group_loop_prefetch(int64_t N, const T* __restrict__ src, T* buf0, Body body) {
+// into a second buffer; otherwise load -> wait -> compute, with the load latency hidden by
+// the other CTAs on the SM.
+template <int P1, int NA, typename T, int NT, int E, int BUF, bool PREFETCH, typename Body>
+__device__ __forceinline__ void group_loop(int64_t N, const T* __restrict__ src, T* buf0, Body body) {
     using G = Geo<P1, NA, T>;
     const int64_t ngroups = (N + E - 1) / E;
-    if constexpr (BC_SPEC_PREFETCH) {
+    if constexpr (PREFETCH) {
         int64_t g = blockIdx.x;
         if (g < ngroups) load_group_async<P1, NA, T, NT>(buf0, src + g * E * G::NPTS, imin64(E, N - g * E));
         cp_async_commit();
@@ -298,10 +295,10 @@ __device__ __forceinline__ void group_loop_prefetch(int64_t N, const T* __restri
 // scalar sum V^2 (R18) is accumulated in the store epilogue: one partial per
 // CTA in ws[8 + blockIdx.x], reduced in fixed order by check_finalize.
 template <int P1, typename T>
-__global__ void __launch_bounds__(Cfg<P1, P1, T, SPEC_NBUF1>::NT)
+__global__ void __launch_bounds__(Cfg<P1, P1, T, 1, K_SF3>::NT)
 sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, const T* __restrict__ C,
                  const T* __restrict__ U, T* __restrict__ V, double* __restrict__ ws) {
-    using CF = Cfg<P1, P1, T, SPEC_NBUF1>;
+    using CF = Cfg<P1, P1, T, 1, K_SF3>;
     using G = Geo<P1, P1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -313,7 +310,7 @@ sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, co
     load_op<P1, T, NT>(opB, B);
     load_op<P1, T, NT>(opC, C);
     double sq = 0.0;
-    group_loop_prefetch<P1, P1, T, NT, CF::E, CF::BUF>(N, U, buf, [&](T* in, int64_t e0, int ne) {
+    group_loop<P1, P1, T, NT, CF::E, CF::BUF, CF::PREFETCH>(N, U, buf, [&](T* in, int64_t e0, int ne) {
         const int nlines = ne * P1 * P1;
         apply_lines<P1, P1, 2, R, NT>(in, opA, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
         __syncthreads();
@@ -330,7 +327,7 @@ sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, co
 
 template <int P1, typename T>
 int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, double* ws, cudaStream_t s) {
-    using CF = Cfg<P1, P1, T, SPEC_NBUF1>;
+    using CF = Cfg<P1, P1, T, 1, K_SF3>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const size_t smem = CF::SMEM + op_elems<P1, T>() * sizeof(T);
@@ -345,11 +342,11 @@ int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, 
 // ====================================================================== sumfact2d
 //   W[l][j] = sum_m A[j][m] U[l][m]  (rows, in place);  V[i][j] = sum_l B[i][l] W[l][j]
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, 1, double, SPEC_NBUF1, K_SF2>::NT)
+__global__ void __launch_bounds__(Cfg<P1, 1, double, 1, K_SF2>::NT)
 sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restrict__ B,
                  const double* __restrict__ U, double* __restrict__ V) {
     using T = double;
-    using CF = Cfg<P1, 1, T, SPEC_NBUF1, K_SF2>;
+    using CF = Cfg<P1, 1, T, 1, K_SF2>;
     using G = Geo<P1, 1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -358,7 +355,7 @@ sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restri
     T* buf = opB + op_elems<P1, T>();
     load_op<P1, T, NT>(opA, A);
     load_op<P1, T, NT>(opB, B);
-    group_loop_prefetch<P1, 1, T, NT, CF::E, CF::BUF>(N, U, buf, [&](T* in, int64_t e0, int ne) {
+    group_loop<P1, 1, T, NT, CF::E, CF::BUF, CF::PREFETCH>(N, U, buf, [&](T* in, int64_t e0, int ne) {
         const int nlines = ne * P1;
         apply_lines<P1, 1, 2, R, NT>(in, opA, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
         __syncthreads();
@@ -371,7 +368,7 @@ sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restri
 
 template <int P1>
 int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* U, double* V, cudaStream_t s) {
-    using CF = Cfg<P1, 1, double, SPEC_NBUF1, K_SF2>;
+    using CF = Cfg<P1, 1, double, 1, K_SF2>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(sumfact2d_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
@@ -384,18 +381,18 @@ int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* 
 // us and ut are stored from registers (coalesced); ur is formed in place (its rows are
 // strided across threads) and copied out coalesced.
 template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, SPEC_NBUF1, K_LG3>::NT)
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 1, K_LG3>::NT)
 local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ U,
                    double* __restrict__ ur, double* __restrict__ us, double* __restrict__ ut) {
     using T = double;
-    using CF = Cfg<P1, P1, T, SPEC_NBUF1, K_LG3>;
+    using CF = Cfg<P1, P1, T, 1, K_LG3>;
     using G = Geo<P1, P1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* opD = reinterpret_cast<T*>(smem_raw);
     T* buf = opD + 2 * op_elems<P1, T>();
     load_op<P1, T, NT>(opD, D);
-    group_loop_prefetch<P1, P1, T, NT, CF::E, CF::BUF>(N, U, buf, [&](T* in, int64_t e0, int ne) {
+    group_loop<P1, P1, T, NT, CF::E, CF::BUF, CF::PREFETCH>(N, U, buf, [&](T* in, int64_t e0, int ne) {
         const int nlines = ne * P1 * P1;
         const int64_t gbase = e0 * G::NPTS;
         apply_lines<P1, P1, 1, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
@@ -415,7 +412,7 @@ local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __rest
 template <int P1>
 int launch_local_grad3(int64_t N, const double* D, const double* U, double* ur, double* us, double* ut,
                        cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, SPEC_NBUF1, K_LG3>;
+    using CF = Cfg<P1, P1, double, 1, K_LG3>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(local_grad3_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
