@@ -550,12 +550,13 @@ static int launch_ccsdt_mma(const CcsdtParams& P, cudaStream_t s) {
 // Each CTA loops over units (a 16^3 hole cube x one particle plane); the unit's t3 values
 // seed the cube (read once, cp.async) and the cube is stored once.
 // Operand layouts in one stage (KC = 8 k values):
-//   d1: A = v2[h3, O2+i2, p6, k] for i2 < 16: 16 copies of [k][h3] (128 B rows, 128B swizzle)
+//   d1: A = v2[h3, O2+i2, p6, k]: 8 copies (h2 pairs) of [k][h2'][h3] (128 B rows, 128B
+//       swizzle; the swizzle row 2k + h2' differs for the 4 k of a fragment)
 //       B = t2[k, p4, p5, h1]: [h1][k] (64 B rows, 64B swizzle)
 //   d2: A = t2[k, p4, h1, h2]: [h2][h1][k] (64 B rows, 64B swizzle)
 //       B = v2[k, h3, p6, p5]: [h3][k] (64 B rows, 64B swizzle)
-// Fragment rows are permuted ({0,1,8,9,2,3,10,11} for the 128B case, {0,1,4,5,2,3,6,7}
-// for the 64B case) so that each half-warp touches 16 distinct banks.
+// 64B-swizzled fragment rows are permuted ({0,1,4,5,2,3,6,7}) so that each half-warp
+// touches 16 distinct banks.
 // ==================================================================================
 struct TmaMaps {
     CUtensorMap a[9];  // d1: v2_v (h3,h2,p6,k) | d2: t2_v (k,p4,h1,h2)
@@ -599,8 +600,7 @@ __device__ __forceinline__ void named_bar_sync(int id, int n) {
     asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(n) : "memory");
 }
 
-// fragment row permutations (see header)
-__device__ __forceinline__ int perm128(int g) { return (g & 1) + 8 * ((g >> 1) & 1) + 2 * (g >> 2); }
+// 64B-swizzle fragment row permutation (see header)
 __device__ __forceinline__ int perm64(int g) { return (g & 1) + 4 * ((g >> 1) & 1) + 2 * (g >> 2); }
 // byte offset of element (row, col) in 64-byte rows under the 64B swizzle
 __device__ __forceinline__ uint32_t swz64(uint32_t row, uint32_t col) {
@@ -670,9 +670,9 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
                 const uint32_t A = st_u32 + slot * TG::STAGE_BYTES;
                 const uint32_t B = A + TG::A_BYTES;
                 if constexpr (FAM == FAM_D1) {
-                    if (lane == 0) {  // one issuing lane measured faster than spreading the 17 copies
+                    if (lane == 0) {  // one issuing lane measured faster than spreading the copies
 #pragma unroll 1
-                        for (int i2 = 0; i2 < 16; ++i2) tma_load_4d(A + i2 * 1024, &M.a[e], O3, O2 + i2, p6, k0, full);
+                        for (int j = 0; j < 8; ++j) tma_load_4d(A + j * 2048, &M.a[e], O3, O2 + 2 * j, p6, k0, full);
                         tma_load_4d(B, &M.b[e], k0, p4, p5, O1, full);
                     }
                 } else {
@@ -744,9 +744,10 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
                 for (int mi = 0; mi < 4; ++mi) {
                     uint32_t off;
                     if constexpr (FAM == FAM_D1) {
-                        const int i2 = 2 * warp + (mi >> 1);
-                        const int i3 = perm128(gq) + 4 * (mi & 1);
-                        off = i2 * 1024 + kk * 128 + ((((i3 >> 1) ^ kk) & 7) << 4) + ((i3 & 1) << 3);
+                        // copy j = warp holds h2 = O2 + 2 warp + {0,1}: rows r = 2 kk + (mi >> 1)
+                        const int i3 = 8 * (mi & 1) + gq;
+                        const int r = 2 * kk + (mi >> 1);
+                        off = warp * 2048 + r * 128 + ((((i3 >> 1) ^ r) & 7) << 4) + ((i3 & 1) << 3);
                     } else {
                         off = swz64(32 * warp + 8 * mi + perm64(gq), kk);
                     }
@@ -776,7 +777,7 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
                     int hi, lo;  // strided pair (lo = fast name, hi = h2)
                     if constexpr (FAM == FAM_D1) {
                         hi = 2 * warp + (mi >> 1);
-                        lo = perm128(gq) + 4 * (mi & 1);
+                        lo = 8 * (mi & 1) + gq;
                     } else {
                         const int sidx = 32 * warp + 8 * mi + perm64(gq);
                         hi = sidx >> 4;
@@ -860,7 +861,7 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
     for (int e = 0; e < P.nentry; ++e) {
         bool ok;
         if (FAM == FAM_D1) {
-            const int da[4] = {H3, H2, P6, K}, ba[4] = {16, 1, 1, TmaGeo::KC};
+            const int da[4] = {H3, H2, P6, K}, ba[4] = {16, 2, 1, TmaGeo::KC};
             const int db[4] = {K, P4, P5, H1}, bb[4] = {TmaGeo::KC, 1, 1, 16};
             ok = encode_4d(&M.a[e], P.opB[e], da, ba, true) && encode_4d(&M.b[e], P.opA[e], db, bb, false);
         } else {
