@@ -85,6 +85,7 @@ struct CcsdtParams {
     const double* opA[9];  // t2 (d1, d2) or t1 (s1), per variant entry
     const double* opB[9];  // v2, per variant entry
     double sign[9];
+    uint32_t smask[9];  // sign as the high-word sign-bit mask (0 or 0x80000000)
     int ppos[9][3];   // per entry: storage position (3..5) of p4, p5, p6
     int ecls[9];      // per entry: class slot
     int hpos[3][3];   // per class slot: storage position (0..2) of h1, h2, h3
@@ -732,7 +733,7 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
             const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
             const unsigned char* B = A + TG::A_BYTES;
             const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
-            const uint32_t smask = P.sign[e] < 0 ? 0x80000000u : 0u;
+            const uint32_t smask = P.smask[e];
 #pragma unroll
             for (int ks = 0; ks < KC / 4; ++ks) {
                 const int kk = ks * 4 + tq;
@@ -937,6 +938,7 @@ int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const
             }
             for (int q = 3; q < 6; ++q) P.ppos[n][vi.order[q] - 3] = q;
             P.sign[n] = vi.sign;
+            P.smask[n] = vi.sign < 0 ? 0x80000000u : 0u;
             P.ecls[n] = ncls;
             P.opA[n] = opA[t];
             P.opB[n] = opB[t];
