@@ -141,6 +141,20 @@ int bc_ccsdt_d2_fused(const bc_tile_dims* d, double* t3, const double* const t2[
 int bc_ccsdt_s1_fused(const bc_tile_dims* d, double* t3, const double* const t1[9],
                       const double* const v2[9], void* stream);
 
+/* All 27 triples variants of one tile block fused, t3 never stored (
+ * P:705-712 "representative of what executes at the socket level"):
+ *     t3 = sum_v s1_v + sum_v d1_v + sum_v d2_v        (from zero, R3/R12/R23)
+ *     ws[0] = E = sum over t3 (canonical order) of t3^2 / (eh3+eh2+eh1-ep6-ep5-ep4)
+ * i.e. bc_check_energy of the t3 that the 27 per-variant calls would build on a zeroed
+ * buffer.  Host arrays of 9 device pointers per list; NULL skips a variant.
+ * Requires h1 = h2 = h3 (even, >= 12), p4 = p5 = p6 and even k (the tile case);
+ * otherwise BC_ERR_UNSUPPORTED.  ws: >= BC_CHECK_WS_DOUBLES doubles. */
+int bc_ccsdt_triples_energy(const bc_tile_dims* d, const double* const t1[9],
+                            const double* const v2s1[9], const double* const t2d1[9],
+                            const double* const v2d1[9], const double* const t2d2[9],
+                            const double* const v2d2[9], const double* eps_h,
+                            const double* eps_p, double* ws, void* stream);
+
 /* North-star convenience form ("trip counts of 16 iterations in each dimension"):
  * all seven extents equal to `tile`. */
 int bc_ccsdt_d1_tile(int variant, int tile, double* t3, const double* t2, const double* v2,

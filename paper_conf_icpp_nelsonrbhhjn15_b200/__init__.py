@@ -21,7 +21,7 @@ from ._abi import BC_CHECK_WS_DOUBLES, TileDims, lib
 
 __all__ = [
     "BarracudaError", "sumfact3d", "sumfact2d", "local_grad3", "local_grad3_t", "ax_e",
-    "ccsdt", "ccsdt_fused", "check_sumsq", "check_energy", "fill", "launch_count",
+    "ccsdt", "ccsdt_fused", "ccsdt_triples_energy", "check_sumsq", "check_energy", "fill", "launch_count",
     "reset_launch_count", "LIB_PATH",
 ]
 
@@ -170,6 +170,28 @@ def ccsdt_fused(family: str, ext, t3: torch.Tensor, t2s, v2s) -> torch.Tensor:
     d = _dims(ext)
     _check(fn(ctypes.byref(d), _dev(t3, f, "t3"), a, b, _stream(t3)), f"bc_ccsdt_{family}_fused")
     return t3
+
+
+def ccsdt_triples_energy(ext, s1, d1, d2, eps_h, eps_p, ws=None) -> torch.Tensor:
+    """Energy of the t3 built from all (non-None) triples variants, t3 never stored.
+    s1 = (t1s, v2s), d1 = (t2s, v2s), d2 = (t2s, v2s): lists of 9 (None = skip).
+    Returns ws[0] (device scalar)."""
+    f = torch.float64
+    dev = eps_h.device
+    if ws is None:
+        ws = torch.empty(BC_CHECK_WS_DOUBLES, dtype=f, device=dev)
+    arrs = []
+    for (xs, ys), nm in ((s1, "s1"), (d1, "d1"), (d2, "d2")):
+        a, b = _abi.PtrArray9(), _abi.PtrArray9()
+        for v in range(9):
+            if xs[v] is not None:
+                a[v] = _dev(xs[v], f, f"{nm}[{v}]")
+                b[v] = _dev(ys[v], f, f"{nm}v2[{v}]")
+        arrs += [a, b]
+    d = _dims(ext)
+    _check(lib.bc_ccsdt_triples_energy(ctypes.byref(d), *arrs, _dev(eps_h, f, "eps_h"), _dev(eps_p, f, "eps_p"),
+                                       _dev(ws, f, "ws"), _stream(eps_h)), "bc_ccsdt_triples_energy")
+    return ws[0]
 
 
 # ----------------------------------------------------------------------------- checks

@@ -21,6 +21,11 @@ int run_sumfact3d_mma(int64_t, int, const double*, const double*, const double*,
                       cudaStream_t);
 int run_sumfact2d_mma(int64_t, int, const double*, const double*, const double*, double*, cudaStream_t);
 int run_local_grad3_mma(int64_t, int, const double*, const double*, double*, double*, double*, cudaStream_t);
+int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const double* const* v2s1,
+                             const double* const* t2d1, const double* const* v2d1, const double* const* t2d2,
+                             const double* const* v2d2, const double* eps_h, const double* eps_p, double* ws,
+                             cudaStream_t s);
+void set_triples_dump(double* p);
 int run_sumsq(int64_t n, const double* x, double* ws, cudaStream_t s);
 int run_energy(const int* ext7, const double* t3, const double* eh, const double* ep, double* ws, cudaStream_t s);
 template <typename T>
@@ -285,6 +290,31 @@ int bc_ccsdt_d2_tile(int variant, int tile, double* t3, const double* t2, const 
     const bc_tile_dims d{tile, tile, tile, tile, tile, tile, tile};
     return ccsdt_one(2, variant, &d, t3, t2, v2, stream);
 }
+
+int bc_ccsdt_triples_energy(const bc_tile_dims* d, const double* const t1[9], const double* const v2s1[9],
+                            const double* const t2d1[9], const double* const v2d1[9], const double* const t2d2[9],
+                            const double* const v2d2[9], const double* eps_h, const double* eps_p, double* ws,
+                            void* stream) {
+    int st = check_dims(d, true);
+    if (st) return st;
+    BC_REQUIRE(t1 && v2s1 && t2d1 && v2d1 && t2d2 && v2d2 && eps_h && eps_p && ws, BC_ERR_ARG);
+    BC_REQUIRE(d->h1 == d->h2 && d->h2 == d->h3 && d->p4 == d->p5 && d->p5 == d->p6, BC_ERR_UNSUPPORTED);
+    BC_REQUIRE(d->k % 2 == 0 && d->h1 % 2 == 0 && d->h1 >= 12, BC_ERR_UNSUPPORTED);
+    BC_REQUIRE(aligned(ws, 8) && aligned(eps_h, 8) && aligned(eps_p, 8), BC_ERR_ALIGN);
+    const double* const* lists[6] = {t1, v2s1, t2d1, v2d1, t2d2, v2d2};
+    for (int l = 0; l < 6; l += 2)
+        for (int v = 0; v < 9; ++v) {
+            if (!lists[l][v]) continue;
+            BC_REQUIRE(lists[l + 1][v] != nullptr, BC_ERR_ARG);
+            BC_REQUIRE(aligned(lists[l][v], 16) && aligned(lists[l + 1][v], 16), BC_ERR_ALIGN);
+        }
+    int e[7];
+    dims_to_ext(d, e, true);
+    return run_ccsdt_triples_energy(e, t1, v2s1, t2d1, v2d1, t2d2, v2d2, eps_h, eps_p, ws, as_stream(stream));
+}
+
+/* debug hook (not in barracuda.h): make bc_ccsdt_triples_energy also store its t3 */
+void bc_debug_triples_dump(double* t3) { set_triples_dump(t3); }
 
 int bc_check_sumsq(int64_t n, const double* x, double* ws, void* stream) {
     BC_REQUIRE(n >= 0 && ws, BC_ERR_ARG);

@@ -609,6 +609,88 @@ __device__ __forceinline__ uint32_t swz64(uint32_t row, uint32_t col) {
     return off ^ (((off >> 7) & 3) << 4);
 }
 
+// ---- per-family pieces shared by the TMA kernels ----------------------------------
+// producer: issue the TMA copies of one (entry e, k chunk k0) stage into slot buffers A/B
+template <int FE>
+__device__ __forceinline__ void tma_issue_stage(const CUtensorMap* ma, const CUtensorMap* mb, uint32_t A, uint32_t B,
+                                                uint32_t full, int lane, int O1, int O2, int O3, int p4, int p5,
+                                                int p6, int k0) {
+    if constexpr (FE == FAM_D1) {
+        if (lane == 0) {  // one issuing lane measured faster than spreading the copies
+#pragma unroll 1
+            for (int j = 0; j < 8; ++j) tma_load_4d(A + j * 2048, ma, O3, O2 + 2 * j, p6, k0, full);
+            tma_load_4d(B, mb, k0, p4, p5, O1, full);
+        }
+    } else {
+        if (lane == 0) tma_load_4d(A, ma, k0, p4, O1, O2, full);
+        if (lane == 1) tma_load_4d(B, mb, k0, O3, p6, p5, full);
+    }
+}
+
+// consumer: one KC = 8 stage of DMMA for this warp's 32 pairs x 16 thirds (k beyond the
+// tensor extent arrives zero-filled by TMA)
+template <int FE>
+__device__ __forceinline__ void tma_consume_stage(const unsigned char* A, const unsigned char* B, uint32_t smask,
+                                                  double (&c)[4][2][2], int warp, int gq, int tq) {
+#pragma unroll
+    for (int ks = 0; ks < TmaGeo::KC / 4; ++ks) {
+        const int kk = ks * 4 + tq;
+        double bf[2], af[4];
+#pragma unroll
+        for (int ni = 0; ni < 2; ++ni)
+            bf[ni] = flip_sign(*reinterpret_cast<const double*>(B + swz64(ni * 8 + perm64(gq), kk)), smask);
+#pragma unroll
+        for (int mi = 0; mi < 4; ++mi) {
+            uint32_t off;
+            if constexpr (FE == FAM_D1) {
+                // copy j = warp holds h2 = O2 + 2 warp + {0,1}: rows r = 2 kk + (mi >> 1)
+                const int i3 = 8 * (mi & 1) + gq;
+                const int r = 2 * kk + (mi >> 1);
+                off = warp * 2048 + r * 128 + ((((i3 >> 1) ^ r) & 7) << 4) + ((i3 & 1) << 3);
+            } else {
+                off = swz64(32 * warp + 8 * mi + perm64(gq), kk);
+            }
+            af[mi] = *reinterpret_cast<const double*>(A + off);
+        }
+#pragma unroll
+        for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+            for (int ni = 0; ni < 2; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[mi], bf[ni]);
+    }
+}
+
+// consumer: add a class's register tile into the accumulator cube at its permuted
+// positions (hp = storage positions of h1, h2, h3) and clear the registers
+template <int FE>
+__device__ __forceinline__ void tma_flush_class(double* acc_s, double (&c)[4][2][2], const int* hp, int warp, int gq,
+                                                int tq) {
+    constexpr int CST = TmaGeo::CST;
+    const int s1 = hp[0] == 0 ? 1 : (hp[0] == 1 ? CST : CST * CST);
+    const int s2 = hp[1] == 0 ? 1 : (hp[1] == 1 ? CST : CST * CST);
+    const int s3 = hp[2] == 0 ? 1 : (hp[2] == 1 ? CST : CST * CST);
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) {
+        int hi, lo;  // strided pair (lo = fast name, hi = h2)
+        if constexpr (FE == FAM_D1) {
+            hi = 2 * warp + (mi >> 1);
+            lo = 8 * (mi & 1) + gq;
+        } else {
+            const int sidx = 32 * warp + 8 * mi + perm64(gq);
+            hi = sidx >> 4;
+            lo = sidx & 15;
+        }
+        const int rowoff = (FE == FAM_D2) ? (lo * s1 + hi * s2) : (lo * s3 + hi * s2);
+        const int sb = (FE == FAM_D2) ? s3 : s1;
+#pragma unroll
+        for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+            for (int j = 0; j < 2; ++j) {
+                acc_s[rowoff + (ni * 8 + perm64(2 * tq + j)) * sb] += c[mi][ni][j];
+                c[mi][ni][j] = 0.0;
+            }
+    }
+}
+
 template <int FAM>
 __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_constant__ CcsdtParams P,
                                                                const __grid_constant__ TmaMaps M, int units) {
@@ -669,17 +751,7 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
                 auto pick = [&](int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
                 const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
                 const uint32_t A = st_u32 + slot * TG::STAGE_BYTES;
-                const uint32_t B = A + TG::A_BYTES;
-                if constexpr (FAM == FAM_D1) {
-                    if (lane == 0) {  // one issuing lane measured faster than spreading the copies
-#pragma unroll 1
-                        for (int j = 0; j < 8; ++j) tma_load_4d(A + j * 2048, &M.a[e], O3, O2 + 2 * j, p6, k0, full);
-                        tma_load_4d(B, &M.b[e], k0, p4, p5, O1, full);
-                    }
-                } else {
-                    if (lane == 0) tma_load_4d(A, &M.a[e], k0, p4, O1, O2, full);
-                    if (lane == 1) tma_load_4d(B, &M.b[e], k0, O3, p6, p5, full);
-                }
+                tma_issue_stage<FAM>(&M.a[e], &M.b[e], A, A + TG::A_BYTES, full, lane, O1, O2, O3, p4, p5, p6, k0);
             }
         }
         return;
@@ -733,67 +805,18 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
             const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
             const unsigned char* B = A + TG::A_BYTES;
             const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
-            const uint32_t smask = P.smask[e];
-#pragma unroll
-            for (int ks = 0; ks < KC / 4; ++ks) {
-                const int kk = ks * 4 + tq;
-                double bf[2], af[4];
-#pragma unroll
-                for (int ni = 0; ni < 2; ++ni)
-                    bf[ni] = flip_sign(*reinterpret_cast<const double*>(B + swz64(ni * 8 + perm64(gq), kk)), smask);
-#pragma unroll
-                for (int mi = 0; mi < 4; ++mi) {
-                    uint32_t off;
-                    if constexpr (FAM == FAM_D1) {
-                        // copy j = warp holds h2 = O2 + 2 warp + {0,1}: rows r = 2 kk + (mi >> 1)
-                        const int i3 = 8 * (mi & 1) + gq;
-                        const int r = 2 * kk + (mi >> 1);
-                        off = warp * 2048 + r * 128 + ((((i3 >> 1) ^ r) & 7) << 4) + ((i3 & 1) << 3);
-                    } else {
-                        off = swz64(32 * warp + 8 * mi + perm64(gq), kk);
-                    }
-                    af[mi] = *reinterpret_cast<const double*>(A + off);
-                }
-#pragma unroll
-                for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-                    for (int ni = 0; ni < 2; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[mi], bf[ni]);
-            }
+            tma_consume_stage<FAM>(A, B, P.smask[e], c, warp, gq, tq);
             __syncwarp();
             if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
             const bool last_chunk = (k0 + KC >= K);
             if (last_chunk && (e + 1 == P.nentry || P.ecls[e + 1] != P.ecls[e])) {
-                if (!seeded) {  // this unit's t3 seed must have landed for everyone
-                    cp_async_wait_n<0>();
-                    named_bar_sync(1, 256);
-                    seeded = true;
-                }
-                const int cl = P.ecls[e];
-                const int h1p = P.hpos[cl][0], h2p = P.hpos[cl][1], h3p = P.hpos[cl][2];
-                const int s1 = h1p == 0 ? 1 : (h1p == 1 ? CST : CST * CST);
-                const int s2 = h2p == 0 ? 1 : (h2p == 1 ? CST : CST * CST);
-                const int s3 = h3p == 0 ? 1 : (h3p == 1 ? CST : CST * CST);
-#pragma unroll
-                for (int mi = 0; mi < 4; ++mi) {
-                    int hi, lo;  // strided pair (lo = fast name, hi = h2)
-                    if constexpr (FAM == FAM_D1) {
-                        hi = 2 * warp + (mi >> 1);
-                        lo = 8 * (mi & 1) + gq;
-                    } else {
-                        const int sidx = 32 * warp + 8 * mi + perm64(gq);
-                        hi = sidx >> 4;
-                        lo = sidx & 15;
-                    }
-                    const int rowoff = (FAM == FAM_D2) ? (lo * s1 + hi * s2) : (lo * s3 + hi * s2);
-                    const int sb = (FAM == FAM_D2) ? s3 : s1;
-#pragma unroll
-                    for (int ni = 0; ni < 2; ++ni)
-#pragma unroll
-                        for (int j = 0; j < 2; ++j) {
-                            acc_s[rowoff + (ni * 8 + perm64(2 * tq + j)) * sb] += c[mi][ni][j];
-                            c[mi][ni][j] = 0.0;
-                        }
-                }
+                // consumer warps only meet at unit boundaries, so without this barrier a fast
+                // warp could flush the next class onto positions a slow warp is still
+                // read-modify-writing for this one (and the seed must have landed)
+                if (!seeded) cp_async_wait_n<0>();
+                seeded = true;
+                named_bar_sync(1, 256);
+                tma_flush_class<FAM>(acc_s, c, P.hpos[P.ecls[e]], warp, gq, tq);
             }
         }
         if (!seeded) {
@@ -884,6 +907,263 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
     const int grid = (int)(units < cap ? units : cap);
     ccsdt_tma_kernel<FAM><<<grid, TmaGeo::NT, TmaGeo::SMEM, s>>>(P, M, (int)units);
     return launch_status();
+}
+
+// ==================================================================================
+// f4: all 27 triples variants of one tile block — d1 and d2 (18 entries)
+// on the tensor cores through the same TMA ring, s1 as rank-1 updates of the cube — into
+// a shared-memory-resident t3 that never touches HBM, followed by the energy epilogue
+// E += t3^2 / (eh3 + eh2 + eh1 - ep6 - ep5 - ep4) over the canonical (h3,h2,h1,p6,p5,p4)
+// positions (the check of R18, here the consumer of t3).  One partial per CTA in
+// ws[8 + blockIdx.x], fixed-order finalize.  Equal hole extents and equal particle
+// extents (the tile case) so all variants share one t3 geometry.
+// ==================================================================================
+constexpr int TRIP_MAXE = 18;
+struct TripParams {
+    int nentry;
+    int efam[TRIP_MAXE], ecls[TRIP_MAXE];
+    uint32_t smask[TRIP_MAXE];
+    int ppos[TRIP_MAXE][3];
+    int hpos[6][3];
+    int ns1;
+    const double* s1t1[9];
+    const double* s1v2[9];
+    double s1sign[9];
+    int s1hpos[9][3], s1ppos[9][3];
+    int ext[7], qe[6], ncube[3];
+    const double* eps_h;
+    const double* eps_p;
+    double* ws;
+    double* dump;  // debug only (bc_debug_triples_dump): store the t3 cube, canonical layout
+};
+struct TripMaps {
+    CUtensorMap a[TRIP_MAXE];
+    CUtensorMap b[TRIP_MAXE];
+};
+
+__global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const __grid_constant__ TripParams P,
+                                                                          const __grid_constant__ TripMaps M,
+                                                                          int units) {
+    using TG = TmaGeo;
+    constexpr int BS = TG::BS, KC = TG::KC, NS = TG::NS, CST = TG::CST;
+    extern __shared__ unsigned char smem_raw[];
+    const uint32_t raw = smem_u32(smem_raw);
+    const uint32_t base = (raw + 1023) & ~1023u;
+    unsigned char* gbase = smem_raw + (base - raw);
+    double* acc_s = reinterpret_cast<double*>(gbase + NS * TG::STAGE_BYTES);
+    const uint32_t bar_full = base + NS * TG::STAGE_BYTES + TG::ACC * 8;
+    const uint32_t bar_empty = bar_full + NS * 8;
+    __shared__ double red[8];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < NS; ++i) {
+            mbar_init(bar_full + 8 * i, 1);
+            mbar_init(bar_empty + 8 * i, TG::NCW);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    __syncthreads();
+    const int ncubes = P.ncube[0] * P.ncube[1] * P.ncube[2];
+    const int K = P.ext[N_K];
+    const int nchunk = (K + KC - 1) / KC;
+    const int nstage = P.nentry * nchunk;
+    auto decode = [&](int u, int* o, int* len, int* qv) {
+        const int cube = u % ncubes, plane = u / ncubes;
+        o[0] = (cube % P.ncube[0]) * BS;
+        o[1] = ((cube / P.ncube[0]) % P.ncube[1]) * BS;
+        o[2] = (cube / (P.ncube[0] * P.ncube[1])) * BS;
+        for (int q = 0; q < 3; ++q) len[q] = min(BS, P.qe[q] - o[q]);
+        qv[0] = plane % P.qe[3];
+        qv[1] = (plane / P.qe[3]) % P.qe[4];
+        qv[2] = plane / (P.qe[3] * P.qe[4]);
+    };
+    auto pick = [](const int* qv, int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
+
+    if (warp == TG::NCW) {
+        int g = 0;
+        for (int u = blockIdx.x; u < units; u += gridDim.x) {
+            int o[3], len[3], qv[3];
+            decode(u, o, len, qv);
+            for (int st = 0; st < nstage; ++st, ++g) {
+                const int slot = g % NS;
+                const uint32_t full = bar_full + 8 * slot;
+                if (lane == 0) {
+                    mbar_wait(bar_empty + 8 * slot, ((g / NS) & 1) ^ 1);
+                    mbar_expect_tx(full, TG::STAGE_BYTES);
+                }
+                __syncwarp();
+                const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+                const int c = P.ecls[e];
+                const int O1 = o[P.hpos[c][0]], O2 = o[P.hpos[c][1]], O3 = o[P.hpos[c][2]];
+                const int p4 = pick(qv, P.ppos[e][0]), p5 = pick(qv, P.ppos[e][1]), p6 = pick(qv, P.ppos[e][2]);
+                const uint32_t A = base + slot * TG::STAGE_BYTES;
+                if (P.efam[e] == FAM_D1)
+                    tma_issue_stage<FAM_D1>(&M.a[e], &M.b[e], A, A + TG::A_BYTES, full, lane, O1, O2, O3, p4, p5, p6, k0);
+                else
+                    tma_issue_stage<FAM_D2>(&M.a[e], &M.b[e], A, A + TG::A_BYTES, full, lane, O1, O2, O3, p4, p5, p6, k0);
+            }
+        }
+        return;
+    }
+
+    const int gq = lane >> 2, tq = lane & 3;
+    const int tid = threadIdx.x;
+    const int H1 = P.ext[N_H1], H2 = P.ext[N_H2], H3 = P.ext[N_H3];
+    const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6];
+    const double* eh1 = P.eps_h;
+    const double* eh2 = P.eps_h + H1;
+    const double* eh3 = P.eps_h + H1 + H2;
+    const double* ep4 = P.eps_p;
+    const double* ep5 = P.eps_p + P4;
+    const double* ep6 = P.eps_p + P4 + P5;
+    double energy = 0.0;
+    int g = 0;
+    for (int u = blockIdx.x; u < units; u += gridDim.x) {
+        int o[3], len[3], qv[3];
+        decode(u, o, len, qv);
+        named_bar_sync(1, 256);  // previous unit's epilogue done with the cube
+        for (int i = tid; i < BS * CST * CST; i += 256) acc_s[i] = 0.0;
+        named_bar_sync(1, 256);
+        double c[4][2][2];
+#pragma unroll
+        for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+            for (int ni = 0; ni < 2; ++ni) c[mi][ni][0] = c[mi][ni][1] = 0.0;
+        for (int st = 0; st < nstage; ++st, ++g) {
+            const int slot = g % NS;
+            mbar_wait(bar_full + 8 * slot, (g / NS) & 1);
+            const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
+            const unsigned char* B = A + TG::A_BYTES;
+            const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+            const bool d1 = P.efam[e] == FAM_D1;
+            if (d1) tma_consume_stage<FAM_D1>(A, B, P.smask[e], c, warp, gq, tq);
+            else tma_consume_stage<FAM_D2>(A, B, P.smask[e], c, warp, gq, tq);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
+            if (k0 + KC >= K && (e + 1 == P.nentry || P.ecls[e + 1] != P.ecls[e])) {
+                named_bar_sync(1, 256);  // no two classes flush concurrently (see ccsdt_tma_kernel)
+                if (d1) tma_flush_class<FAM_D1>(acc_s, c, P.hpos[P.ecls[e]], warp, gq, tq);
+                else tma_flush_class<FAM_D2>(acc_s, c, P.hpos[P.ecls[e]], warp, gq, tq);
+            }
+        }
+        named_bar_sync(1, 256);  // all d1/d2 classes flushed
+        // s1 rank-1 updates and the energy of every cube position this thread owns
+        const int q0 = tid & 15, q1 = tid >> 4;
+        for (int q2 = 0; q2 < BS; ++q2) {
+            if (q0 >= len[0] || q1 >= len[1] || q2 >= len[2]) continue;
+            const int ql[3] = {q0, q1, q2};
+            double t = acc_s[q0 + CST * (q1 + CST * q2)];
+            for (int v = 0; v < P.ns1; ++v) {
+                const int h1 = o[P.s1hpos[v][0]] + ql[P.s1hpos[v][0]];
+                const int h2 = o[P.s1hpos[v][1]] + ql[P.s1hpos[v][1]];
+                const int h3 = o[P.s1hpos[v][2]] + ql[P.s1hpos[v][2]];
+                const int p4 = pick(qv, P.s1ppos[v][0]), p5 = pick(qv, P.s1ppos[v][1]), p6 = pick(qv, P.s1ppos[v][2]);
+                const double a = __ldg(P.s1t1[v] + p4 + (int64_t)P4 * h1);
+                const double b = __ldg(P.s1v2[v] + h3 + (int64_t)H3 * (h2 + (int64_t)H2 * (p6 + (int64_t)P6 * p5)));
+                t += P.s1sign[v] * (a * b);
+            }
+            // canonical order (h3, h2, h1, p6, p5, p4) = storage positions 0..5
+            const double den = ((((eh3[o[0] + q0] + eh2[o[1] + q1]) + eh1[o[2] + q2]) - ep6[qv[0]]) - ep5[qv[1]]) -
+                               ep4[qv[2]];
+            energy += t * t / den;
+            if (P.dump)
+                P.dump[(o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * ((o[2] + q2) +
+                       (int64_t)P.qe[2] * (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]))))] = t;
+        }
+    }
+    // consumer-only block reduction (the producer warp has left)
+    for (int off = 16; off > 0; off >>= 1) energy += __shfl_xor_sync(0xffffffffu, energy, off);
+    if (lane == 0) red[warp] = energy;
+    named_bar_sync(1, 256);
+    if (tid == 0) {
+        double sum = 0.0;
+        for (int w = 0; w < TG::NCW; ++w) sum += red[w];
+        P.ws[8 + blockIdx.x] = sum;
+    }
+}
+
+static double* g_triples_dump = nullptr;  // debug only
+void set_triples_dump(double* p) { g_triples_dump = p; }
+
+// Host: d1/d2 entries grouped by class (d1 classes 0-2, d2 classes 3-5), s1 list.
+int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const double* const* v2s1,
+                             const double* const* t2d1, const double* const* v2d1, const double* const* t2d2,
+                             const double* const* v2d2, const double* eps_h, const double* eps_p, double* ws,
+                             cudaStream_t s) {
+    TripParams P;
+    memset(&P, 0, sizeof(P));
+    TripMaps M;
+    memset(&M, 0, sizeof(M));
+    for (int q = 0; q < 7; ++q) P.ext[q] = ext7[q];
+    const int H = ext7[N_H1], PP = ext7[N_P4], K = ext7[N_K];
+    for (int q = 0; q < 3; ++q) P.qe[q] = H;
+    for (int q = 3; q < 6; ++q) P.qe[q] = PP;
+    for (int q = 0; q < 3; ++q) P.ncube[q] = (H + 15) / 16;
+    P.eps_h = eps_h;
+    P.eps_p = eps_p;
+    P.ws = ws;
+    P.dump = g_triples_dump;
+    int n = 0, ncls = 0;
+    const double* const* tA[2] = {t2d1, t2d2};
+    const double* const* vB[2] = {v2d1, v2d2};
+    for (int f = 0; f < 2; ++f) {
+        const int fam = f == 0 ? FAM_D1 : FAM_D2;
+        for (int cls = 0; cls < 3; ++cls) {
+            bool any = false;
+            for (int v = 1; v <= 9; ++v) {
+                if ((v - 1) % 3 != cls || !tA[f][v - 1]) continue;
+                const VariantInfo vi = variant_info(fam, v);
+                if (!any) {
+                    for (int q = 0; q < 3; ++q) P.hpos[ncls][vi.order[q]] = q;
+                    any = true;
+                }
+                for (int q = 3; q < 6; ++q) P.ppos[n][vi.order[q] - 3] = q;
+                P.efam[n] = fam;
+                P.ecls[n] = ncls;
+                P.smask[n] = vi.sign < 0 ? 0x80000000u : 0u;
+                bool ok;
+                if (fam == FAM_D1) {
+                    const int da[4] = {H, H, PP, K}, ba[4] = {16, 2, 1, TmaGeo::KC};
+                    const int db[4] = {K, PP, PP, H}, bb[4] = {TmaGeo::KC, 1, 1, 16};
+                    ok = encode_4d(&M.a[n], vB[f][v - 1], da, ba, true) && encode_4d(&M.b[n], tA[f][v - 1], db, bb, false);
+                } else {
+                    const int da[4] = {K, PP, H, H}, ba[4] = {TmaGeo::KC, 1, 16, 16};
+                    const int db[4] = {K, H, PP, PP}, bb[4] = {TmaGeo::KC, 16, 1, 1};
+                    ok = encode_4d(&M.a[n], tA[f][v - 1], da, ba, false) && encode_4d(&M.b[n], vB[f][v - 1], db, bb, false);
+                }
+                if (!ok) return BC_ERR_UNSUPPORTED;
+                ++n;
+            }
+            if (any) ++ncls;
+        }
+    }
+    P.nentry = n;
+    int ns = 0;
+    for (int v = 1; v <= 9; ++v) {
+        if (!t1[v - 1]) continue;
+        const VariantInfo vi = variant_info(FAM_S1, v);
+        for (int q = 0; q < 3; ++q) P.s1hpos[ns][vi.order[q]] = q;
+        for (int q = 3; q < 6; ++q) P.s1ppos[ns][vi.order[q] - 3] = q;
+        P.s1sign[ns] = vi.sign;
+        P.s1t1[ns] = t1[v - 1];
+        P.s1v2[ns] = v2s1[v - 1];
+        ++ns;
+    }
+    P.ns1 = ns;
+    static int occ = 0;
+    if (occ == 0) {
+        cudaFuncSetAttribute(ccsdt_triples_energy_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TmaGeo::SMEM);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_triples_energy_kernel, TmaGeo::NT, TmaGeo::SMEM);
+        if (occ < 1) occ = 1;
+    }
+    const int units = P.ncube[0] * P.ncube[1] * P.ncube[2] * PP * PP * PP;
+    int grid = num_sms() * occ;
+    if (grid > units) grid = units;
+    if (grid > CHECK_MAX_PARTIALS) grid = CHECK_MAX_PARTIALS;
+    ccsdt_triples_energy_kernel<<<grid, TmaGeo::NT, TmaGeo::SMEM, s>>>(P, M, units);
+    const int st = launch_status();
+    if (st) return st;
+    return run_check_finalize(grid, ws, s);
 }
 
 // ------------------------------------------------------------------------------------ host

@@ -100,3 +100,57 @@ def test_energy_check(bc):
     got = float(bc.check_energy(ext, to_dev(t3), to_dev(eh), to_dev(ep)).item())
     ref = oracle.energy(ext, t3, eh, ep)
     assert abs(got - ref) <= 1e-12 * abs(ref)
+
+
+@pytest.mark.parametrize("ext", [(16,) * 7, (20, 20, 20, 4, 4, 4, 6)])
+@pytest.mark.parametrize("mask", ["all", "some"])
+def test_triples_energy_f4(bc, ext, mask):
+    """f4: all 27 variants fused, t3 never stored, energy epilogue == oracle energy of the t3
+    built by the 27 per-variant oracle calls on a zeroed buffer.  Bound: |dE| <=
+    sum 2|t3| dt3 / |den| with dt3 = 1e-12 * S (R14) plus the summation rounding of E."""
+    H, P = ext[0], ext[3]
+    fams = {}
+    for fam, base in (("s1", 50), ("d1", 20), ("d2", 20 + 200000)):
+        na, nb = sizes(fam, ext)
+        xs = [syn.tensor(base + v, (na,)) for v in range(1, 10)]
+        ys = [syn.tensor(base + 20 + v, (nb,)) for v in range(1, 10)]
+        if mask == "some":
+            keep = {"s1": (1, 4), "d1": (2, 5, 9), "d2": (1, 6, 7, 8)}[fam]
+            xs = [x if v in keep else None for v, x in enumerate(xs, 1)]
+        fams[fam] = (xs, ys)
+    eh = syn.tensor(60, (3 * H,), kind=syn.KIND_RANGE, lo=-2.0, hi=-0.5)
+    ep = syn.tensor(61, (3 * P,), kind=syn.KIND_RANGE, lo=0.5, hi=2.0)
+    t3 = np.zeros(n3(ext))
+    S = np.zeros(n3(ext))
+    for fam in ("s1", "d1", "d2"):
+        xs, ys = fams[fam]
+        t3 = oracle.ccsdt_fused(fam, ext, t3, xs, ys)
+        S += oracle.ccsdt_abs_bound(fam, ext, np.zeros(n3(ext)), xs, ys)
+    E = oracle.energy(ext, t3, eh, ep)
+    # per-element bound: 2 |t3| * 1e-12 S / |den|; computed with the oracle's energy on |t3|*S
+    bound_t = 2.0 * 1e-12 * abs(oracle.energy(ext, np.sqrt(np.abs(t3) * S), eh, ep))
+    tol = bound_t + 1e-14 * abs(E) + 1e-300
+    dv = lambda xs: [None if x is None else to_dev(x) for x in xs]
+    got = bc.ccsdt_triples_energy(ext, *((dv(fams[f][0]), dv(fams[f][1])) for f in ("s1", "d1", "d2")),
+                                  to_dev(eh), to_dev(ep)).item()
+    assert abs(got - E) <= tol, (got, E, tol)
+
+
+@pytest.mark.parametrize("family", ["d1", "d2"])
+@pytest.mark.parametrize("ext", [(16, 16, 16, 3, 3, 3, 8), (20, 20, 20, 4, 4, 4, 6)])
+def test_tma_short_classes_no_flush_race(bc, family, ext):
+    """Regression: on the warp-specialised TMA path consumer warps meet only at unit
+    boundaries; with one k-chunk and one entry per class a fast warp used to flush the next
+    class onto cube positions a slow warp was still updating (lost updates).  Integer data,
+    bitwise, repeated."""
+    na, nb = sizes(family, ext)
+    t3 = syn.tensor(10, (n3(ext),), kind=syn.KIND_INT)
+    t2s = [syn.tensor(20 + v, (na,), kind=syn.KIND_INT) for v in range(1, 10)]
+    v2s = [syn.tensor(40 + v, (nb,), kind=syn.KIND_INT) for v in range(1, 10)]
+    for mask in ((1, 2, 3), (1, 5, 9), tuple(range(1, 10))):
+        a = [t2s[v - 1] if v in mask else None for v in range(1, 10)]
+        ref = oracle.ccsdt_fused(family, ext, t3, a, v2s)
+        for _ in range(3):
+            d3 = to_dev(t3)
+            bc.ccsdt_fused(family, ext, d3, [None if x is None else to_dev(x) for x in a], [to_dev(x) for x in v2s])
+            assert np.array_equal(to_host(d3), ref), f"{family} {ext} mask={mask}"

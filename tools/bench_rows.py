@@ -151,6 +151,13 @@ def main():
         ms, mean = timed(lambda: bc.ccsdt_fused("s1", ext, t3, t1s, ops["d1"][1]), reps=10)
         emit("ccsdt_s1_fused", f"f3 tile={t} 9 variants fused", ms, mean, 9 * 2.0 * n3, 16.0 * n3 + 9 * 8.0 * (t * t + t ** 4),
              1, "tiles_per_s")
+        eh = bc.fill(torch.empty(3 * t, dtype=torch.float64, device=DEV), 60, kind=bc.KIND_RANGE, lo=-2.0, hi=-0.5)
+        ep = bc.fill(torch.empty(3 * t, dtype=torch.float64, device=DEV), 61, kind=bc.KIND_RANGE, lo=0.5, hi=2.0)
+        ws = torch.empty(1024, dtype=torch.float64, device=DEV)
+        ms, mean = timed(lambda: bc.ccsdt_triples_energy(ext, (t1s, ops["d1"][1]), ops["d1"], ops["d2"], eh, ep, ws),
+                         reps=10)
+        emit("ccsdt_triples_energy", f"f4 tile={t} 27 variants + energy, t3 never stored", ms, mean,
+             (36.0 * t + 18.0 + 4.0) * n3, 9 * 8.0 * (t * t + t ** 4) + 18 * 16.0 * t ** 4, 1, "tiles_per_s")
         del t3, ops, t1s
         torch.cuda.empty_cache()
 
