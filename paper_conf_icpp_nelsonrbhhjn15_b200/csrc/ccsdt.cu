@@ -954,6 +954,7 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const 
     const uint32_t bar_full = base + NS * TG::STAGE_BYTES + TG::ACC * 8;
     const uint32_t bar_empty = bar_full + NS * 8;
     __shared__ double red[8];
+    __shared__ double s1v[256], s1t[16];  // s1 slices of the current variant
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
         for (int i = 0; i < NS; ++i) {
@@ -1047,22 +1048,35 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const 
             }
         }
         named_bar_sync(1, 256);  // all d1/d2 classes flushed
-        // s1 rank-1 updates and the energy of every cube position this thread owns
+        // s1 rank-1 updates t3 += s t1[p4,h1] v2[h3,h2,p6,p5]: per variant the unit needs a
+        // 16x16 (h3,h2) slice of v2 and 16 h1 values of t1, staged in shared memory
         const int q0 = tid & 15, q1 = tid >> 4;
+        for (int v = 0; v < P.ns1; ++v) {
+            const int hp1 = P.s1hpos[v][0], hp2 = P.s1hpos[v][1], hp3 = P.s1hpos[v][2];
+            const int p4 = pick(qv, P.s1ppos[v][0]), p5 = pick(qv, P.s1ppos[v][1]), p6 = pick(qv, P.s1ppos[v][2]);
+            {   // stage: s1v[i2*16 + i3] = v2[O3+i3, O2+i2, p6, p5]; s1t[i1] = s * t1[p4, O1+i1]
+                const int O2 = o[hp2], O3 = o[hp3], O1 = o[hp1];
+                const int i3 = tid & 15, i2 = tid >> 4;
+                const bool ok = O3 + i3 < H3 && O2 + i2 < H2;
+                s1v[tid] = ok ? __ldg(P.s1v2[v] + (O3 + i3) + (int64_t)H3 * ((O2 + i2) + (int64_t)H2 * (p6 + (int64_t)P6 * p5))) : 0.0;
+                if (tid < 16) s1t[tid] = (O1 + tid < H1) ? P.s1sign[v] * __ldg(P.s1t1[v] + p4 + (int64_t)P4 * (O1 + tid)) : 0.0;
+            }
+            named_bar_sync(1, 256);
+            // this thread's positions (q0, q1, q2 = 0..15): local hole indices by the class map
+#pragma unroll 4
+            for (int q2 = 0; q2 < BS; ++q2) {
+                const int ql0 = q0, ql1 = q1, ql2 = q2;
+                const int i1 = hp1 == 0 ? ql0 : (hp1 == 1 ? ql1 : ql2);
+                const int i2 = hp2 == 0 ? ql0 : (hp2 == 1 ? ql1 : ql2);
+                const int i3 = hp3 == 0 ? ql0 : (hp3 == 1 ? ql1 : ql2);
+                acc_s[q0 + CST * (q1 + CST * q2)] += s1t[i1] * s1v[i2 * 16 + i3];
+            }
+            named_bar_sync(1, 256);
+        }
+        // energy of every cube position this thread owns (canonical (h3,h2,h1,p6,p5,p4))
         for (int q2 = 0; q2 < BS; ++q2) {
             if (q0 >= len[0] || q1 >= len[1] || q2 >= len[2]) continue;
-            const int ql[3] = {q0, q1, q2};
-            double t = acc_s[q0 + CST * (q1 + CST * q2)];
-            for (int v = 0; v < P.ns1; ++v) {
-                const int h1 = o[P.s1hpos[v][0]] + ql[P.s1hpos[v][0]];
-                const int h2 = o[P.s1hpos[v][1]] + ql[P.s1hpos[v][1]];
-                const int h3 = o[P.s1hpos[v][2]] + ql[P.s1hpos[v][2]];
-                const int p4 = pick(qv, P.s1ppos[v][0]), p5 = pick(qv, P.s1ppos[v][1]), p6 = pick(qv, P.s1ppos[v][2]);
-                const double a = __ldg(P.s1t1[v] + p4 + (int64_t)P4 * h1);
-                const double b = __ldg(P.s1v2[v] + h3 + (int64_t)H3 * (h2 + (int64_t)H2 * (p6 + (int64_t)P6 * p5)));
-                t += P.s1sign[v] * (a * b);
-            }
-            // canonical order (h3, h2, h1, p6, p5, p4) = storage positions 0..5
+            const double t = acc_s[q0 + CST * (q1 + CST * q2)];
             const double den = ((((eh3[o[0] + q0] + eh2[o[1] + q1]) + eh1[o[2] + q2]) - ep6[qv[0]]) - ep5[qv[1]]) -
                                ep4[qv[2]];
             energy += t * t / den;
