@@ -632,13 +632,17 @@ __device__ __forceinline__ void tma_issue_stage(const CUtensorMap* ma, const CUt
 template <int FE>
 __device__ __forceinline__ void tma_consume_stage(const unsigned char* A, const unsigned char* B, uint32_t smask,
                                                   double (&c)[4][2][2], int warp, int gq, int tq) {
+    double bfa[TmaGeo::KC / 4][2];
+#pragma unroll
+    for (int ks = 0; ks < TmaGeo::KC / 4; ++ks)
+#pragma unroll
+        for (int ni = 0; ni < 2; ++ni)
+            bfa[ks][ni] = flip_sign(*reinterpret_cast<const double*>(B + swz64(ni * 8 + perm64(gq), ks * 4 + tq)), smask);
 #pragma unroll
     for (int ks = 0; ks < TmaGeo::KC / 4; ++ks) {
         const int kk = ks * 4 + tq;
-        double bf[2], af[4];
-#pragma unroll
-        for (int ni = 0; ni < 2; ++ni)
-            bf[ni] = flip_sign(*reinterpret_cast<const double*>(B + swz64(ni * 8 + perm64(gq), kk)), smask);
+        double af[4];
+        const double* bf = bfa[ks];
 #pragma unroll
         for (int mi = 0; mi < 4; ++mi) {
             uint32_t off;
@@ -799,24 +803,37 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
 #pragma unroll
             for (int ni = 0; ni < 2; ++ni) c[mi][ni][0] = c[mi][ni][1] = 0.0;
 
+        // per-entry values cached in registers (dynamic-index constant-bank loads every stage
+        // showed up as long-scoreboard stalls)
+        int e = 0, kc_i = 0;
+        uint32_t smask = P.smask[0];
+        bool class_end = (P.nentry == 1) || (P.ecls[1] != P.ecls[0]);
         for (int st = 0; st < nstage; ++st, ++g) {
             const int slot = g % NS;
             mbar_wait(bar_full + 8 * slot, (g / NS) & 1);
             const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
             const unsigned char* B = A + TG::A_BYTES;
-            const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
-            tma_consume_stage<FAM>(A, B, P.smask[e], c, warp, gq, tq);
+            tma_consume_stage<FAM>(A, B, smask, c, warp, gq, tq);
             __syncwarp();
             if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
-            const bool last_chunk = (k0 + KC >= K);
-            if (last_chunk && (e + 1 == P.nentry || P.ecls[e + 1] != P.ecls[e])) {
+            const bool last_chunk = (++kc_i == nchunk);
+            const int e_cur = e;
+            if (last_chunk) {
+                kc_i = 0;
+                ++e;
+            }
+            if (last_chunk && class_end) {
                 // consumer warps only meet at unit boundaries, so without this barrier a fast
                 // warp could flush the next class onto positions a slow warp is still
                 // read-modify-writing for this one (and the seed must have landed)
                 if (!seeded) cp_async_wait_n<0>();
                 seeded = true;
                 named_bar_sync(1, 256);
-                tma_flush_class<FAM>(acc_s, c, P.hpos[P.ecls[e]], warp, gq, tq);
+                tma_flush_class<FAM>(acc_s, c, P.hpos[P.ecls[e_cur]], warp, gq, tq);
+            }
+            if (last_chunk && e < P.nentry) {
+                smask = P.smask[e];
+                class_end = (e + 1 == P.nentry) || (P.ecls[e + 1] != P.ecls[e]);
             }
         }
         if (!seeded) {
