@@ -927,6 +927,301 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
 }
 
 // ==================================================================================
+// Tile-24 path (hole extents in (16, 24], d1/d2): the same warp-specialised TMA/DMMA
+// scheme on a 24-cube, so a tile-24 block is 24^3 particle planes of one exact cube each
+// (a 16-cube covers 24 as 16 + 8 and computes 2.37x the useful volume).  One CTA per SM:
+// a 24x25x601-strided fp64 cube (115 KB) + a 3-deep ring of KC = 8 stages (37.5 KiB).
+// 12 consumer warps; warp w owns the hole pairs with h2 in {2w, 2w+1}: 6 m-tiles x 3
+// n-tiles of the third hole.
+// Measured on B200 (profiles/): the TMA unit costs ~70 clk per box + ~3.3 clk per
+// box row, so stages are few boxes of long rows (KC = 8 -> 64 B rows where k is
+// innermost in global memory).  Stage layouts:
+//   d2 A = t2[k, p4, h1, h2]: one box {8, 1, 24, 24} -> [h2][h1][k] (64 B rows, 64B swizzle);
+//        m-tile rows pair = 8 mt + perm64(gq): (h1, h2) = (8 (mt % 3) + perm64(gq), mt / 3)
+//   B    = t2[k, p4, p5, h1] (d1) | v2[k, h3, p6, p5] (d2): one box -> [third][k] (64B swizzle)
+//   d1 A = v2[h3, h2, p6, k] (k outermost in global memory), BC_D1_ONEBOX selects:
+//        1: one box {24, 24, 1, 8} -> [k][h2][h3] (the 4 k of a fragment share a bank:
+//           4-way conflicted reads, one TMA box);  m-tile (h3, h2) = (8 (mi % 3) + gq, 2w + mi / 3)
+//        0: 36 boxes {8 h3, 2 h2, 1, 8 k}, 64B swizzle, rows r = 2k + h2' (the swizzle row
+//           carries k: conflict-free);  m-tile (h3, h2) = (8 bx + 4 hx + gq / 2, 2w + gq % 2)
+// ==================================================================================
+#ifndef BC_D1_ONEBOX
+#define BC_D1_ONEBOX 1
+#endif
+struct Tma24Geo {
+    static constexpr int BS = 24, KC = 8, NS = 3, NCW = 12, NT = (NCW + 1) * 32, NCT = NCW * 32;
+    static constexpr int A_BYTES = 576 * KC * 8;          // 36 KiB
+    static constexpr int B_BYTES = BS * KC * 8;           // 1.5 KiB
+    static constexpr int STAGE_BYTES = A_BYTES + B_BYTES; // 38400 = 75 * 512 (64B-swizzle alignment)
+    static constexpr int C1 = 25, C2 = 601;               // cube strides of q1, q2 (q0: 1)
+    static constexpr int ACC = (BS - 1) * (1 + C1 + C2) + 2;  // doubles (even)
+    static constexpr size_t SMEM = 1024 + (size_t)NS * STAGE_BYTES + (size_t)ACC * 8 + 2 * NS * 8;
+};
+
+template <int FAM>
+__global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __grid_constant__ CcsdtParams P,
+                                                                      const __grid_constant__ TmaMaps M, int units) {
+    using TG = Tma24Geo;
+    constexpr int BS = TG::BS, KC = TG::KC, NS = TG::NS;
+    constexpr bool ONEBOX = BC_D1_ONEBOX != 0;
+    extern __shared__ unsigned char smem_raw[];
+    const uint32_t raw = smem_u32(smem_raw);
+    const uint32_t base = (raw + 1023) & ~1023u;
+    unsigned char* gbase = smem_raw + (base - raw);
+    double* acc_s = reinterpret_cast<double*>(gbase + NS * TG::STAGE_BYTES);
+    const uint32_t bar_full = base + NS * TG::STAGE_BYTES + TG::ACC * 8;
+    const uint32_t bar_empty = bar_full + NS * 8;
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < NS; ++i) {
+            mbar_init(bar_full + 8 * i, 1);
+            mbar_init(bar_empty + 8 * i, TG::NCW);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    __syncthreads();
+
+    const int ncubes = P.ncube[0] * P.ncube[1] * P.ncube[2];
+    const int K = P.ext[N_K];
+    const int nchunk = (K + KC - 1) / KC;
+    const int nstage = P.nentry * nchunk;
+    auto decode = [&](int u, int* o, int* len, int* qv) {
+        const int cube = u % ncubes, plane = u / ncubes;
+        o[0] = (cube % P.ncube[0]) * BS;
+        o[1] = ((cube / P.ncube[0]) % P.ncube[1]) * BS;
+        o[2] = (cube / (P.ncube[0] * P.ncube[1])) * BS;
+        for (int q = 0; q < 3; ++q) len[q] = min(BS, P.qe[q] - o[q]);
+        qv[0] = plane % P.qe[3];
+        qv[1] = (plane / P.qe[3]) % P.qe[4];
+        qv[2] = plane / (P.qe[3] * P.qe[4]);
+    };
+
+    if (warp == TG::NCW) {
+        // ================================ producer: lane 0 arms the stage, lanes issue copies
+        int g = 0;
+        for (int u = blockIdx.x; u < units; u += gridDim.x) {
+            int o[3], len[3], qv[3];
+            decode(u, o, len, qv);
+            for (int st = 0; st < nstage; ++st, ++g) {
+                const int slot = g % NS;
+                const uint32_t full = bar_full + 8 * slot;
+                if (lane == 0) {
+                    mbar_wait(bar_empty + 8 * slot, ((g / NS) & 1) ^ 1);
+                    mbar_expect_tx(full, TG::STAGE_BYTES);
+                }
+                __syncwarp();
+                const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+                const int c = P.ecls[e];
+                const int O1 = o[P.hpos[c][0]], O2 = o[P.hpos[c][1]], O3 = o[P.hpos[c][2]];
+                auto pick = [&](int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
+                const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
+                const uint32_t A = base + slot * TG::STAGE_BYTES;
+                const uint32_t B = A + TG::A_BYTES;
+                if constexpr (FAM == FAM_D1) {
+                    if constexpr (ONEBOX) {
+                        if (lane == 0) tma_load_4d(A, &M.a[e], O3, O2, p6, k0, full);
+                    } else {
+                        for (int cp = lane; cp < 36; cp += 32) {
+                            const int by = cp / 3, bx = cp - 3 * (cp / 3);
+                            tma_load_4d(A + cp * 1024, &M.a[e], O3 + 8 * bx, O2 + 2 * by, p6, k0, full);
+                        }
+                    }
+                    if (lane == 1) tma_load_4d(B, &M.b[e], k0, p4, p5, O1, full);
+                } else {
+                    if (lane == 0) tma_load_4d(A, &M.a[e], k0, p4, O1, O2, full);
+                    if (lane == 1) tma_load_4d(B, &M.b[e], k0, O3, p6, p5, full);
+                }
+            }
+        }
+        return;
+    }
+
+    // ==================================== consumers (warps 0..11)
+    const int gq = lane >> 2, tq = lane & 3;
+    const int tid = threadIdx.x;  // < NCT
+    const int Q0 = P.qe[0], Q1 = P.qe[1];
+    // per-lane fragment byte offsets within a stage, k-step ks adds ks * dA / dB
+    uint32_t offA[6];
+    int lo_m[6], h2_m[6];  // this lane's pair (lo, h2) per m-tile
+#pragma unroll
+    for (int mi = 0; mi < 6; ++mi) {
+        if constexpr (FAM == FAM_D1 && ONEBOX) {
+            h2_m[mi] = 2 * warp + mi / 3;
+            lo_m[mi] = 8 * (mi % 3) + gq;
+            offA[mi] = (uint32_t)((tq * 576 + h2_m[mi] * 24 + lo_m[mi]) * 8);
+        } else if constexpr (FAM == FAM_D1) {
+            const int bx = mi >> 1, hx = mi & 1;
+            h2_m[mi] = 2 * warp + (gq & 1);
+            lo_m[mi] = 8 * bx + 4 * hx + (gq >> 1);
+            offA[mi] = (uint32_t)((3 * warp + bx) * 1024);  // + swizzled (row 2k + h2', col) per k-step
+        } else {
+            const int mt = 6 * warp + mi;
+            h2_m[mi] = mt / 3;
+            lo_m[mi] = 8 * (mt % 3) + perm64(gq);
+            offA[mi] = 0;  // swz64(8 mt + perm64(gq), k) per k-step
+        }
+    }
+    int g = 0;
+    for (int u = blockIdx.x; u < units; u += gridDim.x) {
+        int o[3], len[3], qv[3];
+        decode(u, o, len, qv);
+        const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
+                              (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
+        const int nvol = len[0] * len[1] * len[2];
+        named_bar_sync(1, TG::NCT);  // the previous unit's store from the cube is complete
+        for (int i = tid; i < nvol; i += TG::NCT) {
+            const int q0 = i % len[0], r = i / len[0];
+            const int q1 = r % len[1], q2 = r / len[1];
+            cp_async_8(acc_s + q0 + TG::C1 * q1 + TG::C2 * q2,
+                       P.t3 + pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)Q1 * (o[2] + q2)));
+        }
+        cp_async_commit();
+        bool seeded = false;
+
+        double c[6][3][2];
+#pragma unroll
+        for (int mi = 0; mi < 6; ++mi)
+#pragma unroll
+            for (int ni = 0; ni < 3; ++ni) c[mi][ni][0] = c[mi][ni][1] = 0.0;
+
+        int e = 0, kc_i = 0;
+        uint32_t smask = P.smask[0];
+        bool class_end = (P.nentry == 1) || (P.ecls[1] != P.ecls[0]);
+        for (int st = 0; st < nstage; ++st, ++g) {
+            const int slot = g % NS;
+            mbar_wait(bar_full + 8 * slot, (g / NS) & 1);
+            const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
+            const unsigned char* B = A + TG::A_BYTES;
+#pragma unroll
+            for (int ks = 0; ks < KC / 4; ++ks) {
+                const int kk = 4 * ks + tq;
+                double bf[3], af[6];
+#pragma unroll
+                for (int ni = 0; ni < 3; ++ni)
+                    bf[ni] = flip_sign(*reinterpret_cast<const double*>(B + swz64(8 * ni + perm64(gq), kk)), smask);
+#pragma unroll
+                for (int mi = 0; mi < 6; ++mi) {
+                    uint32_t off;
+                    if constexpr (FAM == FAM_D1 && ONEBOX) {
+                        off = offA[mi] + ks * 4 * 576 * 8;
+                    } else if constexpr (FAM == FAM_D1) {
+                        const uint32_t lo = (uint32_t)((2 * kk + (gq & 1)) * 64 + (4 * (mi & 1) + (gq >> 1)) * 8);
+                        off = offA[mi] + (lo ^ (((lo >> 7) & 3) << 4));
+                    } else {
+                        off = swz64(8 * (6 * warp + mi) + perm64(gq), kk);
+                    }
+                    af[mi] = *reinterpret_cast<const double*>(A + off);
+                }
+#pragma unroll
+                for (int mi = 0; mi < 6; ++mi)
+#pragma unroll
+                    for (int ni = 0; ni < 3; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[mi], bf[ni]);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
+            const bool last_chunk = (++kc_i == nchunk);
+            const int e_cur = e;
+            if (last_chunk) {
+                kc_i = 0;
+                ++e;
+            }
+            if (last_chunk && class_end) {
+                if (!seeded) cp_async_wait_n<0>();
+                seeded = true;
+                named_bar_sync(1, TG::NCT);  // one class in flight at a time (see ccsdt_tma_kernel)
+                const int* hp = P.hpos[P.ecls[e_cur]];
+                const int s1 = hp[0] == 0 ? 1 : (hp[0] == 1 ? TG::C1 : TG::C2);
+                const int s2 = hp[1] == 0 ? 1 : (hp[1] == 1 ? TG::C1 : TG::C2);
+                const int s3 = hp[2] == 0 ? 1 : (hp[2] == 1 ? TG::C1 : TG::C2);
+                const int slo = (FAM == FAM_D1) ? s3 : s1;  // lo = h3 (d1) | h1 (d2)
+                const int sth = (FAM == FAM_D1) ? s1 : s3;  // third = h1 (d1) | h3 (d2)
+#pragma unroll
+                for (int mi = 0; mi < 6; ++mi) {
+                    double* row = acc_s + lo_m[mi] * slo + h2_m[mi] * s2;
+#pragma unroll
+                    for (int ni = 0; ni < 3; ++ni)
+#pragma unroll
+                        for (int j = 0; j < 2; ++j) {
+                            row[(8 * ni + perm64(2 * tq + j)) * sth] += c[mi][ni][j];
+                            c[mi][ni][j] = 0.0;
+                        }
+                }
+            }
+            if (last_chunk && e < P.nentry) {
+                smask = P.smask[e];
+                class_end = (e + 1 == P.nentry) || (P.ecls[e + 1] != P.ecls[e]);
+            }
+        }
+        if (!seeded) cp_async_wait_n<0>();
+        named_bar_sync(1, TG::NCT);  // all flushes into this cube are done
+        for (int i = tid; i < nvol; i += TG::NCT) {
+            const int q0 = i % len[0], r = i / len[0];
+            const int q1 = r % len[1], q2 = r / len[1];
+            P.t3[pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)Q1 * (o[2] + q2))] =
+                acc_s[q0 + TG::C1 * q1 + TG::C2 * q2];
+        }
+    }
+    cp_async_wait_all();
+}
+
+static bool encode_4d_sw(CUtensorMap* m, const double* ptr, const int* dims, const int* box, CUtensorMapSwizzle sw) {
+    auto enc = get_encode();
+    if (!enc) return false;
+    cuuint64_t gdim[4], gstr[3];
+    cuuint32_t bdim[4], estr[4] = {1, 1, 1, 1};
+    cuuint64_t st = 8;
+    for (int i = 0; i < 4; ++i) {
+        gdim[i] = (cuuint64_t)dims[i];
+        bdim[i] = (cuuint32_t)box[i];
+        if (i > 0) gstr[i - 1] = st;
+        st *= (cuuint64_t)dims[i];
+    }
+    const CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<double*>(ptr), gdim, gstr, bdim, estr,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
+// returns 1 when the TMA path is unavailable (caller falls back)
+template <int FAM>
+static int launch_ccsdt_tma24(const CcsdtParams& P, cudaStream_t s) {
+    TmaMaps M;
+    memset(&M, 0, sizeof(M));
+    const int H1 = P.ext[N_H1], H2 = P.ext[N_H2], H3 = P.ext[N_H3];
+    const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6], K = P.ext[N_K];
+    constexpr int KC = Tma24Geo::KC;
+    for (int e = 0; e < P.nentry; ++e) {
+        bool ok;
+        if (FAM == FAM_D1) {
+            const int da[4] = {H3, H2, P6, K}, db[4] = {K, P4, P5, H1}, bb[4] = {KC, 1, 1, 24};
+            const int ba1[4] = {24, 24, 1, KC}, ba0[4] = {8, 2, 1, KC};
+            ok = (BC_D1_ONEBOX ? encode_4d_sw(&M.a[e], P.opB[e], da, ba1, CU_TENSOR_MAP_SWIZZLE_NONE)
+                               : encode_4d_sw(&M.a[e], P.opB[e], da, ba0, CU_TENSOR_MAP_SWIZZLE_64B)) &&
+                 encode_4d_sw(&M.b[e], P.opA[e], db, bb, CU_TENSOR_MAP_SWIZZLE_64B);
+        } else {
+            const int da[4] = {K, P4, H1, H2}, ba[4] = {KC, 1, 24, 24};
+            const int db[4] = {K, H3, P6, P5}, bb[4] = {KC, 24, 1, 1};
+            ok = encode_4d_sw(&M.a[e], P.opA[e], da, ba, CU_TENSOR_MAP_SWIZZLE_64B) &&
+                 encode_4d_sw(&M.b[e], P.opB[e], db, bb, CU_TENSOR_MAP_SWIZZLE_64B);
+        }
+        if (!ok) return 1;
+    }
+    static int occ = 0;
+    if (occ == 0) {
+        cudaFuncSetAttribute(ccsdt_tma24_kernel<FAM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Tma24Geo::SMEM);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_tma24_kernel<FAM>, Tma24Geo::NT, Tma24Geo::SMEM);
+        if (occ < 1) occ = 1;
+    }
+    const int64_t units = (int64_t)P.ncube[0] * P.ncube[1] * P.ncube[2] * P.qe[3] * P.qe[4] * P.qe[5];
+    if (units == 0) return BC_OK;
+    const int64_t cap = (int64_t)num_sms() * occ;
+    const int grid = (int)(units < cap ? units : cap);
+    ccsdt_tma24_kernel<FAM><<<grid, Tma24Geo::NT, Tma24Geo::SMEM, s>>>(P, M, (int)units);
+    return launch_status();
+}
+
+// ==================================================================================
 // f4: all 27 triples variants of one tile block — d1 and d2 (18 entries)
 // on the tensor cores through the same TMA ring, s1 as rank-1 updates of the cube — into
 // a shared-memory-resident t3 that never touches HBM, followed by the energy epilogue
@@ -1264,6 +1559,19 @@ int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const
     // cubes zero-filled by TMA): measured 2x faster than the 12-cube DFMA kernel at tile 24.
     const bool tc_shape = (fam != FAM_S1) && (ext7[N_K] % 2 == 0) && (fam != FAM_D1 || ext7[N_H3] % 2 == 0) &&
                           P.qe[0] >= 12 && P.qe[1] >= 12 && P.qe[2] >= 12 && getenv("BC_NO_MMA") == nullptr;
+    // 24-cube TMA path when its padded hole volume is smaller than the 16-cube's (tile 24)
+    if (tc_shape && getenv("BC_NO_TMA") == nullptr && getenv("BC_NO_TMA24") == nullptr) {
+        long v16 = 1, v24 = 1;
+        for (int q = 0; q < 3; ++q) {
+            v16 *= (long)((P.qe[q] + 15) / 16) * 16;
+            v24 *= (long)((P.qe[q] + 23) / 24) * 24;
+        }
+        if (v24 < v16) {
+            for (int q = 0; q < 3; ++q) P.ncube[q] = (P.qe[q] + 23) / 24;
+            const int st = (fam == FAM_D1) ? launch_ccsdt_tma24<FAM_D1>(P, s) : launch_ccsdt_tma24<FAM_D2>(P, s);
+            if (st != 1) return st;
+        }
+    }
     const int bs = tc_shape ? 16 : choose_bs(P.qe);
     for (int q = 0; q < 3; ++q) P.ncube[q] = (P.qe[q] + bs - 1) / bs;
     const bool mma_ok = bs == 16 && tc_shape;

@@ -65,6 +65,29 @@ def test_fused_integer_bitwise(bc, family, ext):
         assert np.array_equal(to_host(d3), oracle.ccsdt_fused(family, ext, t3, a, v2s)), f"{family} mask={list(mask)}"
 
 
+# hole extents in (16, 24] take the 24-cube TMA path (ccsdt_tma24_kernel): unequal holes, a
+# ragged k chunk (10 = 4 + 4 + 2), a second ragged cube (40 = 24 + 16), exact 24-cubes
+EXTS24 = [(18, 22, 24, 3, 2, 4, 10), (24, 24, 40, 2, 2, 3, 8), (24, 20, 22, 2, 3, 2, 6)]
+
+
+@pytest.mark.parametrize("family", ["d1", "d2"])
+@pytest.mark.parametrize("ext", EXTS24)
+def test_tile24_path_integer_bitwise(bc, family, ext):
+    na, nb = sizes(family, ext)
+    t3 = syn.tensor(10, (n3(ext),), kind=syn.KIND_INT)
+    t2s = [syn.tensor(20 + v, (na,), kind=syn.KIND_INT) for v in range(1, 10)]
+    v2s = [syn.tensor(40 + v, (nb,), kind=syn.KIND_INT) for v in range(1, 10)]
+    for v in (1, 2, 3, 5, 9):
+        d3 = to_dev(t3)
+        bc.ccsdt(family, v, ext, d3, to_dev(t2s[v - 1]), to_dev(v2s[v - 1]))
+        assert np.array_equal(to_host(d3), oracle.ccsdt(family, v, ext, t3, t2s[v - 1], v2s[v - 1])), f"{family}_{v}"
+    for mask in (range(1, 10), (2, 4, 9)):
+        a = [t2s[v - 1] if v in mask else None for v in range(1, 10)]
+        d3 = to_dev(t3)
+        bc.ccsdt_fused(family, ext, d3, [None if x is None else to_dev(x) for x in a], [to_dev(x) for x in v2s])
+        assert np.array_equal(to_host(d3), oracle.ccsdt_fused(family, ext, t3, a, v2s)), f"{family} mask={list(mask)}"
+
+
 @pytest.mark.parametrize("family", ["d1", "d2"])
 @pytest.mark.parametrize("tile", [16, 24])
 def test_tile_random_tolerance(bc, family, tile):
