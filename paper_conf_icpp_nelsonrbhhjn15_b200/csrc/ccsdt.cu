@@ -601,6 +601,16 @@ __device__ __forceinline__ void named_bar_sync(int id, int n) {
     asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(n) : "memory");
 }
 
+// fragment loads as volatile asm: kept in program order relative to the (volatile) DMMAs,
+// so a stage's fragments are all loaded into distinct registers before its first DMMA
+// (plain loads let ptxas reuse one register per fragment and expose the LDS latency
+// between DMMAs)
+__device__ __forceinline__ double lds64(const void* p) {
+    double v;
+    asm volatile("ld.shared.f64 %0, [%1];\n" : "=d"(v) : "r"(smem_u32(p)));
+    return v;
+}
+
 // 64B-swizzle fragment row permutation (see header)
 __device__ __forceinline__ int perm64(int g) { return (g & 1) + 4 * ((g >> 1) & 1) + 2 * (g >> 2); }
 // byte offset of element (row, col) in 64-byte rows under the 64B swizzle
@@ -632,17 +642,14 @@ __device__ __forceinline__ void tma_issue_stage(const CUtensorMap* ma, const CUt
 template <int FE>
 __device__ __forceinline__ void tma_consume_stage(const unsigned char* A, const unsigned char* B, uint32_t smask,
                                                   double (&c)[4][2][2], int warp, int gq, int tq) {
-    double bfa[TmaGeo::KC / 4][2];
+    double bfa[TmaGeo::KC / 4][2], afa[TmaGeo::KC / 4][4];
 #pragma unroll
     for (int ks = 0; ks < TmaGeo::KC / 4; ++ks)
 #pragma unroll
-        for (int ni = 0; ni < 2; ++ni)
-            bfa[ks][ni] = flip_sign(*reinterpret_cast<const double*>(B + swz64(ni * 8 + perm64(gq), ks * 4 + tq)), smask);
+        for (int ni = 0; ni < 2; ++ni) bfa[ks][ni] = lds64(B + swz64(ni * 8 + perm64(gq), ks * 4 + tq));
 #pragma unroll
     for (int ks = 0; ks < TmaGeo::KC / 4; ++ks) {
         const int kk = ks * 4 + tq;
-        double af[4];
-        const double* bf = bfa[ks];
 #pragma unroll
         for (int mi = 0; mi < 4; ++mi) {
             uint32_t off;
@@ -654,13 +661,19 @@ __device__ __forceinline__ void tma_consume_stage(const unsigned char* A, const 
             } else {
                 off = swz64(32 * warp + 8 * mi + perm64(gq), kk);
             }
-            af[mi] = *reinterpret_cast<const double*>(A + off);
+            afa[ks][mi] = lds64(A + off);
         }
+    }
+#pragma unroll
+    for (int ks = 0; ks < TmaGeo::KC / 4; ++ks)
+#pragma unroll
+        for (int ni = 0; ni < 2; ++ni) bfa[ks][ni] = flip_sign(bfa[ks][ni], smask);
+#pragma unroll
+    for (int ks = 0; ks < TmaGeo::KC / 4; ++ks)
 #pragma unroll
         for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
-            for (int ni = 0; ni < 2; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[mi], bf[ni]);
-    }
+            for (int ni = 0; ni < 2; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], afa[ks][mi], bfa[ks][ni]);
 }
 
 // consumer: add a class's register tile into the accumulator cube at its permuted
@@ -931,25 +944,21 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
 // scheme on a 24-cube, so a tile-24 block is 24^3 particle planes of one exact cube each
 // (a 16-cube covers 24 as 16 + 8 and computes 2.37x the useful volume).  One CTA per SM:
 // a 24x25x601-strided fp64 cube (115 KB) + a 3-deep ring of KC = 8 stages (37.5 KiB).
-// 12 consumer warps; warp w owns the hole pairs with h2 in {2w, 2w+1}: 6 m-tiles x 3
-// n-tiles of the third hole.
-// Measured on B200 (profiles/): the TMA unit costs ~70 clk per box + ~3.3 clk per
-// box row, so stages are few boxes of long rows (KC = 8 -> 64 B rows where k is
-// innermost in global memory).  Stage layouts:
-//   d2 A = t2[k, p4, h1, h2]: one box {8, 1, 24, 24} -> [h2][h1][k] (64 B rows, 64B swizzle);
-//        m-tile rows pair = 8 mt + perm64(gq): (h1, h2) = (8 (mt % 3) + perm64(gq), mt / 3)
-//   B    = t2[k, p4, p5, h1] (d1) | v2[k, h3, p6, p5] (d2): one box -> [third][k] (64B swizzle)
-//   d1 A = v2[h3, h2, p6, k] (k outermost in global memory), BC_D1_ONEBOX selects:
-//        1: one box {24, 24, 1, 8} -> [k][h2][h3] (the 4 k of a fragment share a bank:
-//           4-way conflicted reads, one TMA box);  m-tile (h3, h2) = (8 (mi % 3) + gq, 2w + mi / 3)
-//        0: 36 boxes {8 h3, 2 h2, 1, 8 k}, 64B swizzle, rows r = 2k + h2' (the swizzle row
-//           carries k: conflict-free);  m-tile (h3, h2) = (8 bx + 4 hx + gq / 2, 2w + gq % 2)
+// 8 consumer warps + 1 producer (at most 3 warps per SM sub-partition: 168 registers, so
+// a stage's 24 fragments stay in distinct registers next to 54 accumulators); warp w owns
+// the hole pairs with h2 in {3w, 3w+1, 3w+2}: 9 m-tiles x 3 n-tiles of the third hole.
+// Measured on B200 (profiles/): the TMA unit costs ~70 clk per box + ~3.3 clk per box
+// row, so a stage is two boxes with long rows.  Stage layouts:
+//   d2 A = t2[k, p4, h1, h2]: box {8, 1, 24, 24} -> [h2][h1][k] (64 B rows, 64B swizzle);
+//        m-tile mt = 9w + mi: rows 8 mt + perm64(gq), (h1, h2) = (8 (mt % 3) + perm64(gq), mt / 3)
+//   d1 A = v2[h3, h2, p6, k] (k outermost in global memory): box {24, 24, 1, 8} ->
+//        [k][h2][h3] (192 B rows; the 4 k of a fragment share a bank: 4-way conflicted
+//        reads, measured faster than 36 conflict-free 64B-swizzled boxes);
+//        m-tile (h3, h2) = (8 (mi % 3) + gq, 3w + mi / 3)
+//   B    = t2[k, p4, p5, h1] (d1) | v2[k, h3, p6, p5] (d2): box -> [third][k] (64B swizzle)
 // ==================================================================================
-#ifndef BC_D1_ONEBOX
-#define BC_D1_ONEBOX 1
-#endif
 struct Tma24Geo {
-    static constexpr int BS = 24, KC = 8, NS = 3, NCW = 12, NT = (NCW + 1) * 32, NCT = NCW * 32;
+    static constexpr int BS = 24, KC = 8, NS = 3, NCW = 8, NT = (NCW + 1) * 32, NCT = NCW * 32;
     static constexpr int A_BYTES = 576 * KC * 8;          // 36 KiB
     static constexpr int B_BYTES = BS * KC * 8;           // 1.5 KiB
     static constexpr int STAGE_BYTES = A_BYTES + B_BYTES; // 38400 = 75 * 512 (64B-swizzle alignment)
@@ -962,8 +971,7 @@ template <int FAM>
 __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __grid_constant__ CcsdtParams P,
                                                                       const __grid_constant__ TmaMaps M, int units) {
     using TG = Tma24Geo;
-    constexpr int BS = TG::BS, KC = TG::KC, NS = TG::NS;
-    constexpr bool ONEBOX = BC_D1_ONEBOX != 0;
+    constexpr int BS = TG::BS, KC = TG::KC, NS = TG::NS, NCT = TG::NCT;
     extern __shared__ unsigned char smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
     const uint32_t base = (raw + 1023) & ~1023u;
@@ -998,7 +1006,7 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
     };
 
     if (warp == TG::NCW) {
-        // ================================ producer: lane 0 arms the stage, lanes issue copies
+        // ================================ producer: lane 0 arms the stage, lanes 0/1 issue A/B
         int g = 0;
         for (int u = blockIdx.x; u < units; u += gridDim.x) {
             int o[3], len[3], qv[3];
@@ -1019,14 +1027,7 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
                 const uint32_t A = base + slot * TG::STAGE_BYTES;
                 const uint32_t B = A + TG::A_BYTES;
                 if constexpr (FAM == FAM_D1) {
-                    if constexpr (ONEBOX) {
-                        if (lane == 0) tma_load_4d(A, &M.a[e], O3, O2, p6, k0, full);
-                    } else {
-                        for (int cp = lane; cp < 36; cp += 32) {
-                            const int by = cp / 3, bx = cp - 3 * (cp / 3);
-                            tma_load_4d(A + cp * 1024, &M.a[e], O3 + 8 * bx, O2 + 2 * by, p6, k0, full);
-                        }
-                    }
+                    if (lane == 0) tma_load_4d(A, &M.a[e], O3, O2, p6, k0, full);
                     if (lane == 1) tma_load_4d(B, &M.b[e], k0, p4, p5, O1, full);
                 } else {
                     if (lane == 0) tma_load_4d(A, &M.a[e], k0, p4, O1, O2, full);
@@ -1037,31 +1038,13 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
         return;
     }
 
-    // ==================================== consumers (warps 0..11)
+    // ==================================== consumers (warps 0..7)
     const int gq = lane >> 2, tq = lane & 3;
     const int tid = threadIdx.x;  // < NCT
     const int Q0 = P.qe[0], Q1 = P.qe[1];
-    // per-lane fragment byte offsets within a stage, k-step ks adds ks * dA / dB
-    uint32_t offA[6];
-    int lo_m[6], h2_m[6];  // this lane's pair (lo, h2) per m-tile
-#pragma unroll
-    for (int mi = 0; mi < 6; ++mi) {
-        if constexpr (FAM == FAM_D1 && ONEBOX) {
-            h2_m[mi] = 2 * warp + mi / 3;
-            lo_m[mi] = 8 * (mi % 3) + gq;
-            offA[mi] = (uint32_t)((tq * 576 + h2_m[mi] * 24 + lo_m[mi]) * 8);
-        } else if constexpr (FAM == FAM_D1) {
-            const int bx = mi >> 1, hx = mi & 1;
-            h2_m[mi] = 2 * warp + (gq & 1);
-            lo_m[mi] = 8 * bx + 4 * hx + (gq >> 1);
-            offA[mi] = (uint32_t)((3 * warp + bx) * 1024);  // + swizzled (row 2k + h2', col) per k-step
-        } else {
-            const int mt = 6 * warp + mi;
-            h2_m[mi] = mt / 3;
-            lo_m[mi] = 8 * (mt % 3) + perm64(gq);
-            offA[mi] = 0;  // swz64(8 mt + perm64(gq), k) per k-step
-        }
-    }
+    // full 24-cubes of a block whose hole extents are 24: the unit's t3 values are one
+    // contiguous run, and thread t owns q0 = t % 24 (NCT = 256: q0 advances by 16 per copy)
+    const bool dense = (P.qe[0] == BS && P.qe[1] == BS && P.qe[2] == BS);
     int g = 0;
     for (int u = blockIdx.x; u < units; u += gridDim.x) {
         int o[3], len[3], qv[3];
@@ -1069,19 +1052,29 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
         const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
                               (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
         const int nvol = len[0] * len[1] * len[2];
-        named_bar_sync(1, TG::NCT);  // the previous unit's store from the cube is complete
-        for (int i = tid; i < nvol; i += TG::NCT) {
-            const int q0 = i % len[0], r = i / len[0];
-            const int q1 = r % len[1], q2 = r / len[1];
-            cp_async_8(acc_s + q0 + TG::C1 * q1 + TG::C2 * q2,
-                       P.t3 + pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)Q1 * (o[2] + q2)));
+        named_bar_sync(1, NCT);  // the previous unit's store from the cube is complete
+        if (dense) {
+            const double* src = P.t3 + pbase;
+#pragma unroll 6
+            for (int i = tid; i < BS * BS * BS; i += NCT) {
+                const int r = i / BS, q0 = i - r * BS;  // constant divisor: multiply-shift
+                const int q2 = r / BS, q1 = r - q2 * BS;
+                cp_async_8(acc_s + q0 + TG::C1 * q1 + TG::C2 * q2, src + i);
+            }
+        } else {
+            for (int i = tid; i < nvol; i += NCT) {
+                const int q0 = i % len[0], r = i / len[0];
+                const int q1 = r % len[1], q2 = r / len[1];
+                cp_async_8(acc_s + q0 + TG::C1 * q1 + TG::C2 * q2,
+                           P.t3 + pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)Q1 * (o[2] + q2)));
+            }
         }
         cp_async_commit();
         bool seeded = false;
 
-        double c[6][3][2];
+        double c[9][3][2];
 #pragma unroll
-        for (int mi = 0; mi < 6; ++mi)
+        for (int mi = 0; mi < 9; ++mi)
 #pragma unroll
             for (int ni = 0; ni < 3; ++ni) c[mi][ni][0] = c[mi][ni][1] = 0.0;
 
@@ -1093,31 +1086,32 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
             mbar_wait(bar_full + 8 * slot, (g / NS) & 1);
             const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
             const unsigned char* B = A + TG::A_BYTES;
+            double bf[KC / 4][3], af[KC / 4][9];
 #pragma unroll
             for (int ks = 0; ks < KC / 4; ++ks) {
                 const int kk = 4 * ks + tq;
-                double bf[3], af[6];
 #pragma unroll
-                for (int ni = 0; ni < 3; ++ni)
-                    bf[ni] = flip_sign(*reinterpret_cast<const double*>(B + swz64(8 * ni + perm64(gq), kk)), smask);
+                for (int ni = 0; ni < 3; ++ni) bf[ks][ni] = lds64(B + swz64(8 * ni + perm64(gq), kk));
 #pragma unroll
-                for (int mi = 0; mi < 6; ++mi) {
+                for (int mi = 0; mi < 9; ++mi) {
                     uint32_t off;
-                    if constexpr (FAM == FAM_D1 && ONEBOX) {
-                        off = offA[mi] + ks * 4 * 576 * 8;
-                    } else if constexpr (FAM == FAM_D1) {
-                        const uint32_t lo = (uint32_t)((2 * kk + (gq & 1)) * 64 + (4 * (mi & 1) + (gq >> 1)) * 8);
-                        off = offA[mi] + (lo ^ (((lo >> 7) & 3) << 4));
-                    } else {
-                        off = swz64(8 * (6 * warp + mi) + perm64(gq), kk);
-                    }
-                    af[mi] = *reinterpret_cast<const double*>(A + off);
+                    if constexpr (FAM == FAM_D1)
+                        off = (uint32_t)((kk * 576 + (3 * warp + mi / 3) * 24 + 8 * (mi % 3) + gq) * 8);
+                    else
+                        off = swz64(8 * (9 * warp + mi) + perm64(gq), kk);
+                    af[ks][mi] = lds64(A + off);
                 }
-#pragma unroll
-                for (int mi = 0; mi < 6; ++mi)
-#pragma unroll
-                    for (int ni = 0; ni < 3; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[mi], bf[ni]);
             }
+#pragma unroll
+            for (int ks = 0; ks < KC / 4; ++ks)
+#pragma unroll
+                for (int ni = 0; ni < 3; ++ni) bf[ks][ni] = flip_sign(bf[ks][ni], smask);
+#pragma unroll
+            for (int ks = 0; ks < KC / 4; ++ks)
+#pragma unroll
+                for (int mi = 0; mi < 9; ++mi)
+#pragma unroll
+                    for (int ni = 0; ni < 3; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[ks][mi], bf[ks][ni]);
             __syncwarp();
             if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
             const bool last_chunk = (++kc_i == nchunk);
@@ -1129,7 +1123,7 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
             if (last_chunk && class_end) {
                 if (!seeded) cp_async_wait_n<0>();
                 seeded = true;
-                named_bar_sync(1, TG::NCT);  // one class in flight at a time (see ccsdt_tma_kernel)
+                named_bar_sync(1, NCT);  // one class in flight at a time (see ccsdt_tma_kernel)
                 const int* hp = P.hpos[P.ecls[e_cur]];
                 const int s1 = hp[0] == 0 ? 1 : (hp[0] == 1 ? TG::C1 : TG::C2);
                 const int s2 = hp[1] == 0 ? 1 : (hp[1] == 1 ? TG::C1 : TG::C2);
@@ -1137,8 +1131,10 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
                 const int slo = (FAM == FAM_D1) ? s3 : s1;  // lo = h3 (d1) | h1 (d2)
                 const int sth = (FAM == FAM_D1) ? s1 : s3;  // third = h1 (d1) | h3 (d2)
 #pragma unroll
-                for (int mi = 0; mi < 6; ++mi) {
-                    double* row = acc_s + lo_m[mi] * slo + h2_m[mi] * s2;
+                for (int mi = 0; mi < 9; ++mi) {
+                    const int h2 = 3 * warp + mi / 3;
+                    const int lo = 8 * (mi % 3) + ((FAM == FAM_D1) ? gq : perm64(gq));
+                    double* row = acc_s + lo * slo + h2 * s2;
 #pragma unroll
                     for (int ni = 0; ni < 3; ++ni)
 #pragma unroll
@@ -1154,12 +1150,22 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
             }
         }
         if (!seeded) cp_async_wait_n<0>();
-        named_bar_sync(1, TG::NCT);  // all flushes into this cube are done
-        for (int i = tid; i < nvol; i += TG::NCT) {
-            const int q0 = i % len[0], r = i / len[0];
-            const int q1 = r % len[1], q2 = r / len[1];
-            P.t3[pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)Q1 * (o[2] + q2))] =
-                acc_s[q0 + TG::C1 * q1 + TG::C2 * q2];
+        named_bar_sync(1, NCT);  // all flushes into this cube are done
+        if (dense) {
+            double* dst = P.t3 + pbase;
+#pragma unroll 6
+            for (int i = tid; i < BS * BS * BS; i += NCT) {
+                const int r = i / BS, q0 = i - r * BS;
+                const int q2 = r / BS, q1 = r - q2 * BS;
+                dst[i] = acc_s[q0 + TG::C1 * q1 + TG::C2 * q2];
+            }
+        } else {
+            for (int i = tid; i < nvol; i += NCT) {
+                const int q0 = i % len[0], r = i / len[0];
+                const int q1 = r % len[1], q2 = r / len[1];
+                P.t3[pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)Q1 * (o[2] + q2))] =
+                    acc_s[q0 + TG::C1 * q1 + TG::C2 * q2];
+            }
         }
     }
     cp_async_wait_all();
@@ -1194,10 +1200,9 @@ static int launch_ccsdt_tma24(const CcsdtParams& P, cudaStream_t s) {
     for (int e = 0; e < P.nentry; ++e) {
         bool ok;
         if (FAM == FAM_D1) {
-            const int da[4] = {H3, H2, P6, K}, db[4] = {K, P4, P5, H1}, bb[4] = {KC, 1, 1, 24};
-            const int ba1[4] = {24, 24, 1, KC}, ba0[4] = {8, 2, 1, KC};
-            ok = (BC_D1_ONEBOX ? encode_4d_sw(&M.a[e], P.opB[e], da, ba1, CU_TENSOR_MAP_SWIZZLE_NONE)
-                               : encode_4d_sw(&M.a[e], P.opB[e], da, ba0, CU_TENSOR_MAP_SWIZZLE_64B)) &&
+            const int da[4] = {H3, H2, P6, K}, ba[4] = {24, 24, 1, KC};
+            const int db[4] = {K, P4, P5, H1}, bb[4] = {KC, 1, 1, 24};
+            ok = encode_4d_sw(&M.a[e], P.opB[e], da, ba, CU_TENSOR_MAP_SWIZZLE_NONE) &&
                  encode_4d_sw(&M.b[e], P.opA[e], db, bb, CU_TENSOR_MAP_SWIZZLE_64B);
         } else {
             const int da[4] = {K, P4, H1, H2}, ba[4] = {KC, 1, 24, 24};
