@@ -943,7 +943,7 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
 // Tile-24 path (hole extents in (16, 24], d1/d2): the same warp-specialised TMA/DMMA
 // scheme on a 24-cube, so a tile-24 block is 24^3 particle planes of one exact cube each
 // (a 16-cube covers 24 as 16 + 8 and computes 2.37x the useful volume).  One CTA per SM:
-// a 24x25x601-strided fp64 cube (115 KB) + a 3-deep ring of KC = 8 stages (37.5 KiB).
+// a (1, 25, 601)-strided fp64 cube (115 KB) + a 3-deep ring of KC = 8 stages (37.5 KiB).
 // 8 consumer warps + 1 producer (at most 3 warps per SM sub-partition: 168 registers, so
 // a stage's 24 fragments stay in distinct registers next to 54 accumulators); warp w owns
 // the hole pairs with h2 in {3w, 3w+1, 3w+2}: 9 m-tiles x 3 n-tiles of the third hole.
@@ -957,6 +957,12 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
 //        m-tile (h3, h2) = (8 (mi % 3) + gq, 3w + mi / 3)
 //   B    = t2[k, p4, p5, h1] (d1) | v2[k, h3, p6, p5] (d2): box -> [third][k] (64B swizzle)
 // ==================================================================================
+#ifndef BC_EXP_NOSEED
+#define BC_EXP_NOSEED 0  // timing experiments only: skip the t3 seed/store
+#endif
+#ifndef BC_EXP_NOFLUSH
+#define BC_EXP_NOFLUSH 0  // timing experiments only: skip the class flushes
+#endif
 struct Tma24Geo {
     static constexpr int BS = 24, KC = 8, NS = 3, NCW = 8, NT = (NCW + 1) * 32, NCT = NCW * 32;
     static constexpr int A_BYTES = 576 * KC * 8;          // 36 KiB
@@ -1053,7 +1059,8 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
                               (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
         const int nvol = len[0] * len[1] * len[2];
         named_bar_sync(1, NCT);  // the previous unit's store from the cube is complete
-        if (dense) {
+        if (BC_EXP_NOSEED) {
+        } else if (dense) {
             const double* src = P.t3 + pbase;
 #pragma unroll 6
             for (int i = tid; i < BS * BS * BS; i += NCT) {
@@ -1078,29 +1085,28 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
 #pragma unroll
             for (int ni = 0; ni < 3; ++ni) c[mi][ni][0] = c[mi][ni][1] = 0.0;
 
-        int e = 0, kc_i = 0;
+        int e = 0, kc_i = 0, cls_stages = 0;
         uint32_t smask = P.smask[0];
         bool class_end = (P.nentry == 1) || (P.ecls[1] != P.ecls[0]);
         for (int st = 0; st < nstage; ++st, ++g) {
+            ++cls_stages;
             const int slot = g % NS;
             mbar_wait(bar_full + 8 * slot, (g / NS) & 1);
             const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
             const unsigned char* B = A + TG::A_BYTES;
             double bf[KC / 4][3], af[KC / 4][9];
+            // one base address per k-step; the m-/n-tiles are immediate offsets (an 8-row
+            // step of a 64B-swizzled operand is 512 B and leaves the XOR pattern unchanged)
 #pragma unroll
             for (int ks = 0; ks < KC / 4; ++ks) {
-                const int kk = 4 * ks + tq;
+                const unsigned char* Bk = B + swz64(perm64(gq), 4 * ks + tq);
+                const unsigned char* Ak = (FAM == FAM_D1) ? A + ((4 * ks + tq) * 576 + 72 * warp + gq) * 8
+                                                          : A + 9 * warp * 512 + swz64(perm64(gq), 4 * ks + tq);
 #pragma unroll
-                for (int ni = 0; ni < 3; ++ni) bf[ks][ni] = lds64(B + swz64(8 * ni + perm64(gq), kk));
+                for (int ni = 0; ni < 3; ++ni) bf[ks][ni] = lds64(Bk + ni * 512);
 #pragma unroll
-                for (int mi = 0; mi < 9; ++mi) {
-                    uint32_t off;
-                    if constexpr (FAM == FAM_D1)
-                        off = (uint32_t)((kk * 576 + (3 * warp + mi / 3) * 24 + 8 * (mi % 3) + gq) * 8);
-                    else
-                        off = swz64(8 * (9 * warp + mi) + perm64(gq), kk);
-                    af[ks][mi] = lds64(A + off);
-                }
+                for (int mi = 0; mi < 9; ++mi)
+                    af[ks][mi] = lds64(Ak + ((FAM == FAM_D1) ? ((mi / 3) * 24 + 8 * (mi % 3)) * 8 : mi * 512));
             }
 #pragma unroll
             for (int ks = 0; ks < KC / 4; ++ks)
@@ -1121,9 +1127,23 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
                 ++e;
             }
             if (last_chunk && class_end) {
+                // CTA-wide barrier before a flush: always before the first (the seed copies of
+                // all threads have landed); before later ones only when the class that just
+                // ends here spans <= NS stages.  Otherwise no warp can reach this flush while
+                // another is still flushing the previous class: the producer refills a slot
+                // only after all consumers released it, so the fastest warp is at most NS
+                // stages ahead of the slowest.
+                const bool need_bar = !seeded || cls_stages <= NS;
                 if (!seeded) cp_async_wait_n<0>();
                 seeded = true;
-                named_bar_sync(1, NCT);  // one class in flight at a time (see ccsdt_tma_kernel)
+                if (need_bar) named_bar_sync(1, NCT);
+                cls_stages = 0;
+                if (BC_EXP_NOFLUSH) {
+#pragma unroll
+                    for (int mi = 0; mi < 9; ++mi)
+#pragma unroll
+                        for (int ni = 0; ni < 3; ++ni) if (c[mi][ni][0] == 1.2345) acc_s[mi] = c[mi][ni][1];
+                } else {
                 const int* hp = P.hpos[P.ecls[e_cur]];
                 const int s1 = hp[0] == 0 ? 1 : (hp[0] == 1 ? TG::C1 : TG::C2);
                 const int s2 = hp[1] == 0 ? 1 : (hp[1] == 1 ? TG::C1 : TG::C2);
@@ -1143,6 +1163,7 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
                             c[mi][ni][j] = 0.0;
                         }
                 }
+                }
             }
             if (last_chunk && e < P.nentry) {
                 smask = P.smask[e];
@@ -1151,7 +1172,8 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
         }
         if (!seeded) cp_async_wait_n<0>();
         named_bar_sync(1, NCT);  // all flushes into this cube are done
-        if (dense) {
+        if (BC_EXP_NOSEED) {
+        } else if (dense) {
             double* dst = P.t3 + pbase;
 #pragma unroll 6
             for (int i = tid; i < BS * BS * BS; i += NCT) {
