@@ -67,7 +67,8 @@ def test_fused_integer_bitwise(bc, family, ext):
 
 # hole extents in (16, 24] take the 24-cube TMA path (ccsdt_tma24_kernel): unequal holes, a
 # ragged k chunk (10 = 4 + 4 + 2), a second ragged cube (40 = 24 + 16), exact 24-cubes
-EXTS24 = [(18, 22, 24, 3, 2, 4, 10), (24, 24, 40, 2, 2, 3, 8), (24, 20, 22, 2, 3, 2, 6)]
+# (24, 24, 24, ...) is a dense block (contiguous t3 runs per unit, division-free seed/store)
+EXTS24 = [(18, 22, 24, 3, 2, 4, 10), (24, 24, 40, 2, 2, 3, 8), (24, 20, 22, 2, 3, 2, 6), (24, 24, 24, 2, 3, 2, 10)]
 
 
 @pytest.mark.parametrize("family", ["d1", "d2"])
