@@ -14,6 +14,11 @@
 
 #include "common.cuh"
 
+// unroll factor of the contracted-index loop (experiments only)
+#ifndef BC_NUNROLL
+#define BC_NUNROLL 1
+#endif
+
 namespace bc {
 
 // ------------------------------------------------------------------------------------
@@ -124,7 +129,7 @@ struct Line {
 // 16-byte broadcast operator load feeds 2R FMAs and there are P1*R independent FMA
 // chains per thread.  All reads of a line precede the writes of that line and every
 // line is read by exactly one thread, so `out` may overwrite the line in place.
-template <int P1, int NA, int AXIS, int R, int NT, typename T, typename Out>
+template <int P1, int NA, int AXIS, int R, int NT, typename T, typename Out, int UNR = BC_NUNROLL>
 __device__ __forceinline__ void apply_lines(const T* in, const T* opT, int nlines, Out out) {
     using G = Geo<P1, NA, T>;
     using LN = Line<P1, NA, AXIS, T>;
@@ -143,7 +148,7 @@ __device__ __forceinline__ void apply_lines(const T* in, const T* opT, int nline
         for (int k = 0; k < P1; ++k)
 #pragma unroll
             for (int r = 0; r < R; ++r) acc[k][r] = T(0);
-#pragma unroll 1
+#pragma unroll UNR
         for (int n = 0; n < P1; ++n) {
             T x[R];
 #pragma unroll
@@ -207,16 +212,36 @@ __host__ __device__ __forceinline__ int imin64(int64_t a, int64_t b) { return (i
 // live field (+1 for the prefetch of the next group).
 // Variant table, measured on B200 with tools/sweep_spectral.py (profiles/sweep_spectral_r01.md):
 //   P1 >= 10: sumfact3d / local_grad3: R = 4 lines per thread, 54 KiB element groups, no
-//             in-CTA prefetch (occupancy hides the loads); sumfact2d: R = 3, 18 KiB groups
-//             with prefetch; local_grad3_t / ax_e: R = 2, 18 KiB.
+//             in-CTA prefetch (occupancy hides the loads), except P1 = 12: R = 3, 36 KiB;
+//             sumfact2d: R = 3, 18 KiB groups with prefetch; local_grad3_t / ax_e: R = 2, 18 KiB.
 //   P1 <  10: R = 2, 18 KiB groups with prefetch (36 KiB for local_grad3).
+//   sumfact2d at P1 >= 9 fully unrolls its contracted-index loop (0.64 -> 0.75 of HBM at P1 = 13).
+//   Rejected (same sweep): n-loop unroll 2 / 13 for sumfact3d and local_grad3 (register
+//   spills), prefetching 18/36 KiB groups at P1 >= 10.
 enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
+// experiment overrides for the P1 >= 10 sumfact3d / local_grad3 entries (variant sweeps only)
+#ifndef BC_BIG_R
+#define BC_BIG_R 4
+#endif
+#ifndef BC_BIG_KB
+#define BC_BIG_KB 54
+#endif
+#ifndef BC_BIG_PF
+#define BC_BIG_PF 0
+#endif
+#ifndef BC_SF2_UNROLL
+#define BC_SF2_UNROLL 1
+#endif
 template <int P1, int KIND>
 struct SpecTable {
     static constexpr bool BIG = P1 >= 10;
-    static constexpr int R = BIG ? (KIND == K_SF3 || KIND == K_LG3 ? 4 : (KIND == K_SF2 ? 3 : 2)) : 2;
-    static constexpr int BUF_KB = BIG ? (KIND == K_SF3 || KIND == K_LG3 ? 54 : 18) : (KIND == K_LG3 ? 36 : 18);
-    static constexpr bool PREFETCH = !(BIG && (KIND == K_SF3 || KIND == K_LG3));
+    static constexpr bool SF3LG3 = KIND == K_SF3 || KIND == K_LG3;
+    static constexpr bool MID = P1 == 12;  // sumfact3d / local_grad3: R = 3, 36 KiB (measured)
+    static constexpr int R = BIG ? (SF3LG3 ? (MID ? 3 : BC_BIG_R) : (KIND == K_SF2 ? 3 : 2)) : 2;
+    static constexpr int BUF_KB = BIG ? (SF3LG3 ? (MID ? 36 : BC_BIG_KB) : 18) : (KIND == K_LG3 ? 36 : 18);
+    static constexpr bool PREFETCH = !(BIG && SF3LG3) || BC_BIG_PF;
+    // unroll of the contracted-index loop: sumfact2d fully (its two stages fit the registers)
+    static constexpr int UNROLL = (KIND == K_SF2 && BC_SF2_UNROLL && P1 >= 9) ? P1 : BC_NUNROLL;
 };
 
 template <int P1, int NA, typename T, int NBUF_FIELDS, int KIND = K_SF3>
@@ -357,12 +382,13 @@ sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restri
     load_op<P1, T, NT>(opB, B);
     group_loop<P1, 1, T, NT, CF::E, CF::BUF, CF::PREFETCH>(N, U, buf, [&](T* in, int64_t e0, int ne) {
         const int nlines = ne * P1;
-        apply_lines<P1, 1, 2, R, NT>(in, opA, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
+        constexpr int U = CF::TB::UNROLL;
+        auto st1 = [&](int, int base, int k, T v) { in[base + k] = v; };
+        apply_lines<P1, 1, 2, R, NT, T, decltype(st1), U>(in, opA, nlines, st1);
         __syncthreads();
         T* Vg = V + e0 * G::NPTS;
-        apply_lines<P1, 1, 1, R, NT>(in, opB, nlines, [&](int L, int, int k, T v) {
-            st_cs(Vg + Line<P1, 1, 1, T>::gofs(L, k), v);
-        });
+        auto st2 = [&](int L, int, int k, T v) { st_cs(Vg + Line<P1, 1, 1, T>::gofs(L, k), v); };
+        apply_lines<P1, 1, 1, R, NT, T, decltype(st2), U>(in, opB, nlines, st2);
     });
 }
 
