@@ -564,12 +564,18 @@ struct TmaMaps {
     CUtensorMap b[9];  // d1: t2_v (k,p4,p5,h1) | d2: v2_v (k,h3,p6,p5)
 };
 
+#ifndef BC_TC16_KC
+#define BC_TC16_KC 16
+#endif
 struct TmaGeo {
-    // two CTAs per SM (measured better than one CTA with a deeper ring), 4-deep ring
-    static constexpr int BS = 16, KC = 8, NS = 4, NCW = 8, NT = (NCW + 1) * 32;
-    static constexpr int A_BYTES = 16 * 16 * KC * 8;  // 16 KiB
-    static constexpr int B_BYTES = 16 * KC * 8;       // 1 KiB
-    static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;  // 17 KiB (multiple of 1 KiB)
+    // two CTAs per SM (measured better than one CTA with a deeper ring).  KC = 8: 64 B
+    // operand rows (64B swizzle), 4-deep ring;  KC = 16: 128 B rows (128B swizzle, half the
+    // TMA rows per byte), 2-deep ring
+    static constexpr int BS = 16, KC = BC_TC16_KC, NS = KC == 16 ? 2 : 4, NCW = 8, NT = (NCW + 1) * 32;
+    static constexpr int A_BYTES = 16 * 16 * KC * 8;  // 16 | 32 KiB
+    static constexpr int B_BYTES = 16 * KC * 8;       // 1 | 2 KiB
+    static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;  // multiple of 1 KiB
+    static constexpr int ROW = KC * 8;                // operand row bytes (k innermost)
     static constexpr int CST = BS + 1;
     static constexpr int ACC = BS * CST * CST;          // doubles
     static constexpr size_t SMEM = 1024 + (size_t)NS * STAGE_BYTES + ACC * 8 + 2 * NS * 8;
@@ -618,17 +624,40 @@ __device__ __forceinline__ uint32_t swz64(uint32_t row, uint32_t col) {
     const uint32_t off = row * 64 + col * 8;
     return off ^ (((off >> 7) & 3) << 4);
 }
+// 16-cube kernels: k-innermost operand rows of TmaGeo::ROW bytes, swizzled (64B | 128B);
+// fragment row permutation so a half-warp's 4 rows x 4 k hit 16 distinct banks, and an
+// 8-row step (+8 ROW bytes) leaves the XOR pattern unchanged
+__device__ __forceinline__ int permK(int g) {
+    return TmaGeo::KC == 16 ? 2 * (g & 3) + (g >> 2) : perm64(g);
+}
+__device__ __forceinline__ uint32_t swzK(uint32_t row, uint32_t col) {
+    if (TmaGeo::KC == 16) {
+        const uint32_t off = row * 128 + col * 8;
+        return off ^ ((row & 7) << 4);
+    }
+    return swz64(row, col);
+}
 
 // ---- per-family pieces shared by the TMA kernels ----------------------------------
+// d1's A slice v2[h3, h2, p6, k] (k outermost in global memory): 1 = one TMA box
+// {16, 16, 1, 8} -> [k][h2][h3] (4-way conflicted fragment reads, 2 boxes per stage);
+// 0 = 8 boxes {16, 2, 1, 8} with 128B swizzle (conflict-free reads, 9 boxes per stage).
+// The TMA unit costs ~70 clk per box + ~3.3 clk per box row (measured).
+#ifndef BC_TC16_ONEBOX
+#define BC_TC16_ONEBOX 0
+#endif
 // producer: issue the TMA copies of one (entry e, k chunk k0) stage into slot buffers A/B
 template <int FE>
 __device__ __forceinline__ void tma_issue_stage(const CUtensorMap* ma, const CUtensorMap* mb, uint32_t A, uint32_t B,
                                                 uint32_t full, int lane, int O1, int O2, int O3, int p4, int p5,
                                                 int p6, int k0) {
-    if constexpr (FE == FAM_D1) {
+    if constexpr (FE == FAM_D1 && BC_TC16_ONEBOX) {
+        if (lane == 0) tma_load_4d(A, ma, O3, O2, p6, k0, full);
+        if (lane == 1) tma_load_4d(B, mb, k0, p4, p5, O1, full);
+    } else if constexpr (FE == FAM_D1) {
         if (lane == 0) {  // one issuing lane measured faster than spreading the copies
 #pragma unroll 1
-            for (int j = 0; j < 8; ++j) tma_load_4d(A + j * 2048, ma, O3, O2 + 2 * j, p6, k0, full);
+            for (int j = 0; j < 8; ++j) tma_load_4d(A + j * (TmaGeo::A_BYTES / 8), ma, O3, O2 + 2 * j, p6, k0, full);
             tma_load_4d(B, mb, k0, p4, p5, O1, full);
         }
     } else {
@@ -643,23 +672,36 @@ template <int FE>
 __device__ __forceinline__ void tma_consume_stage(const unsigned char* A, const unsigned char* B, uint32_t smask,
                                                   double (&c)[4][2][2], int warp, int gq, int tq) {
     double bfa[TmaGeo::KC / 4][2], afa[TmaGeo::KC / 4][4];
+    // an 8-row step of a 64B-swizzled operand is +512 B with the same XOR pattern, so the
+    // n-/m-tiles are immediate offsets from one base per k-step
 #pragma unroll
-    for (int ks = 0; ks < TmaGeo::KC / 4; ++ks)
+    for (int ks = 0; ks < TmaGeo::KC / 4; ++ks) {
+        const unsigned char* Bk = B + swzK(permK(gq), ks * 4 + tq);
 #pragma unroll
-        for (int ni = 0; ni < 2; ++ni) bfa[ks][ni] = lds64(B + swz64(ni * 8 + perm64(gq), ks * 4 + tq));
+        for (int ni = 0; ni < 2; ++ni) bfa[ks][ni] = lds64(Bk + ni * 8 * TmaGeo::ROW);
+    }
 #pragma unroll
     for (int ks = 0; ks < TmaGeo::KC / 4; ++ks) {
         const int kk = ks * 4 + tq;
+        const unsigned char* Ak = (FE == FAM_D1) ? A + (kk * 256 + 32 * warp + gq) * 8
+                                                 : A + 32 * warp * TmaGeo::ROW + swzK(permK(gq), kk);
 #pragma unroll
         for (int mi = 0; mi < 4; ++mi) {
             uint32_t off;
-            if constexpr (FE == FAM_D1) {
+            if constexpr (FE == FAM_D1 && BC_TC16_ONEBOX) {
+                // one box [k][h2][h3]: pair (h3, h2) = (8 (mi & 1) + gq, 2 warp + (mi >> 1))
+                afa[ks][mi] = lds64(Ak + ((mi >> 1) * 16 + 8 * (mi & 1)) * 8);
+                continue;
+            } else if constexpr (FE == FAM_D2) {
+                afa[ks][mi] = lds64(Ak + mi * 8 * TmaGeo::ROW);
+                continue;
+            } else if constexpr (FE == FAM_D1) {
                 // copy j = warp holds h2 = O2 + 2 warp + {0,1}: rows r = 2 kk + (mi >> 1)
                 const int i3 = 8 * (mi & 1) + gq;
                 const int r = 2 * kk + (mi >> 1);
-                off = warp * 2048 + r * 128 + ((((i3 >> 1) ^ r) & 7) << 4) + ((i3 & 1) << 3);
+                off = warp * (TmaGeo::A_BYTES / 8) + r * 128 + ((((i3 >> 1) ^ r) & 7) << 4) + ((i3 & 1) << 3);
             } else {
-                off = swz64(32 * warp + 8 * mi + perm64(gq), kk);
+                off = swzK(32 * warp + 8 * mi + permK(gq), kk);
             }
             afa[ks][mi] = lds64(A + off);
         }
@@ -692,7 +734,7 @@ __device__ __forceinline__ void tma_flush_class(double* acc_s, double (&c)[4][2]
             hi = 2 * warp + (mi >> 1);
             lo = 8 * (mi & 1) + gq;
         } else {
-            const int sidx = 32 * warp + 8 * mi + perm64(gq);
+            const int sidx = 32 * warp + 8 * mi + permK(gq);
             hi = sidx >> 4;
             lo = sidx & 15;
         }
@@ -702,7 +744,7 @@ __device__ __forceinline__ void tma_flush_class(double* acc_s, double (&c)[4][2]
         for (int ni = 0; ni < 2; ++ni)
 #pragma unroll
             for (int j = 0; j < 2; ++j) {
-                acc_s[rowoff + (ni * 8 + perm64(2 * tq + j)) * sb] += c[mi][ni][j];
+                acc_s[rowoff + (ni * 8 + permK(2 * tq + j)) * sb] += c[mi][ni][j];
                 c[mi][ni][j] = 0.0;
             }
     }
@@ -818,10 +860,11 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
 
         // per-entry values cached in registers (dynamic-index constant-bank loads every stage
         // showed up as long-scoreboard stalls)
-        int e = 0, kc_i = 0;
+        int e = 0, kc_i = 0, cls_stages = 0;
         uint32_t smask = P.smask[0];
         bool class_end = (P.nentry == 1) || (P.ecls[1] != P.ecls[0]);
         for (int st = 0; st < nstage; ++st, ++g) {
+            ++cls_stages;
             const int slot = g % NS;
             mbar_wait(bar_full + 8 * slot, (g / NS) & 1);
             const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
@@ -838,10 +881,15 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
             if (last_chunk && class_end) {
                 // consumer warps only meet at unit boundaries, so without this barrier a fast
                 // warp could flush the next class onto positions a slow warp is still
-                // read-modify-writing for this one (and the seed must have landed)
+                // read-modify-writing for this one (and the seed must have landed).  Not
+                // needed after the first flush when the class spans more than NS stages: the
+                // producer refills a slot only after all consumers released it, so the
+                // fastest warp is at most NS stages ahead of the slowest.
+                const bool need_bar = !seeded || cls_stages <= NS;
                 if (!seeded) cp_async_wait_n<0>();
                 seeded = true;
-                named_bar_sync(1, 256);
+                if (need_bar) named_bar_sync(1, 256);
+                cls_stages = 0;
                 tma_flush_class<FAM>(acc_s, c, P.hpos[P.ecls[e_cur]], warp, gq, tq);
             }
             if (last_chunk && e < P.nentry) {
@@ -887,7 +935,7 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
     return fn;
 }
 
-static bool encode_4d(CUtensorMap* m, const double* ptr, const int* dims, const int* box, bool swz128) {
+static bool encode_4d_sw(CUtensorMap* m, const double* ptr, const int* dims, const int* box, CUtensorMapSwizzle sw) {
     auto enc = get_encode();
     if (!enc) return false;
     cuuint64_t gdim[4], gstr[3];
@@ -900,9 +948,20 @@ static bool encode_4d(CUtensorMap* m, const double* ptr, const int* dims, const 
         st *= (cuuint64_t)dims[i];
     }
     const CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<double*>(ptr), gdim, gstr, bdim, estr,
-                           CU_TENSOR_MAP_INTERLEAVE_NONE, swz128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
-                           CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
+}
+
+static bool encode_4d(CUtensorMap* m, const double* ptr, const int* dims, const int* box, bool swz128) {
+    return encode_4d_sw(m, ptr, dims, box, swz128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B);
+}
+
+// d1 A (v2) tensor map of the 16-cube kernels (see BC_TC16_ONEBOX)
+static bool encode_d1_a16(CUtensorMap* m, const double* v2, const int* dims) {
+    const int one[4] = {16, 16, 1, TmaGeo::KC}, eight[4] = {16, 2, 1, TmaGeo::KC};
+    return BC_TC16_ONEBOX ? encode_4d_sw(m, v2, dims, one, CU_TENSOR_MAP_SWIZZLE_NONE)
+                          : encode_4d_sw(m, v2, dims, eight, CU_TENSOR_MAP_SWIZZLE_128B);
 }
 
 // returns 1 when the TMA path is unavailable (caller falls back)
@@ -915,13 +974,14 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
     for (int e = 0; e < P.nentry; ++e) {
         bool ok;
         if (FAM == FAM_D1) {
-            const int da[4] = {H3, H2, P6, K}, ba[4] = {16, 2, 1, TmaGeo::KC};
+            const int da[4] = {H3, H2, P6, K};
             const int db[4] = {K, P4, P5, H1}, bb[4] = {TmaGeo::KC, 1, 1, 16};
-            ok = encode_4d(&M.a[e], P.opB[e], da, ba, true) && encode_4d(&M.b[e], P.opA[e], db, bb, false);
+            ok = encode_d1_a16(&M.a[e], P.opB[e], da) && encode_4d(&M.b[e], P.opA[e], db, bb, TmaGeo::KC == 16);
         } else {
             const int da[4] = {K, P4, H1, H2}, ba[4] = {TmaGeo::KC, 1, 16, 16};
             const int db[4] = {K, H3, P6, P5}, bb[4] = {TmaGeo::KC, 16, 1, 1};
-            ok = encode_4d(&M.a[e], P.opA[e], da, ba, false) && encode_4d(&M.b[e], P.opB[e], db, bb, false);
+            ok = encode_4d(&M.a[e], P.opA[e], da, ba, TmaGeo::KC == 16) &&
+                 encode_4d(&M.b[e], P.opB[e], db, bb, TmaGeo::KC == 16);
         }
         if (!ok) return 1;
     }
@@ -1193,23 +1253,6 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
     cp_async_wait_all();
 }
 
-static bool encode_4d_sw(CUtensorMap* m, const double* ptr, const int* dims, const int* box, CUtensorMapSwizzle sw) {
-    auto enc = get_encode();
-    if (!enc) return false;
-    cuuint64_t gdim[4], gstr[3];
-    cuuint32_t bdim[4], estr[4] = {1, 1, 1, 1};
-    cuuint64_t st = 8;
-    for (int i = 0; i < 4; ++i) {
-        gdim[i] = (cuuint64_t)dims[i];
-        bdim[i] = (cuuint32_t)box[i];
-        if (i > 0) gstr[i - 1] = st;
-        st *= (cuuint64_t)dims[i];
-    }
-    const CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<double*>(ptr), gdim, gstr, bdim, estr,
-                           CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    return r == CUDA_SUCCESS;
-}
 
 // returns 1 when the TMA path is unavailable (caller falls back)
 template <int FAM>
@@ -1476,13 +1519,15 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
                 P.smask[n] = vi.sign < 0 ? 0x80000000u : 0u;
                 bool ok;
                 if (fam == FAM_D1) {
-                    const int da[4] = {H, H, PP, K}, ba[4] = {16, 2, 1, TmaGeo::KC};
+                    const int da[4] = {H, H, PP, K};
                     const int db[4] = {K, PP, PP, H}, bb[4] = {TmaGeo::KC, 1, 1, 16};
-                    ok = encode_4d(&M.a[n], vB[f][v - 1], da, ba, true) && encode_4d(&M.b[n], tA[f][v - 1], db, bb, false);
+                    ok = encode_d1_a16(&M.a[n], vB[f][v - 1], da) &&
+                         encode_4d(&M.b[n], tA[f][v - 1], db, bb, TmaGeo::KC == 16);
                 } else {
                     const int da[4] = {K, PP, H, H}, ba[4] = {TmaGeo::KC, 1, 16, 16};
                     const int db[4] = {K, H, PP, PP}, bb[4] = {TmaGeo::KC, 16, 1, 1};
-                    ok = encode_4d(&M.a[n], tA[f][v - 1], da, ba, false) && encode_4d(&M.b[n], vB[f][v - 1], db, bb, false);
+                    ok = encode_4d(&M.a[n], tA[f][v - 1], da, ba, TmaGeo::KC == 16) &&
+                         encode_4d(&M.b[n], vB[f][v - 1], db, bb, TmaGeo::KC == 16);
                 }
                 if (!ok) return BC_ERR_UNSUPPORTED;
                 ++n;
