@@ -129,6 +129,13 @@ __device__ __forceinline__ void cp_async_8_zfill(void* dst, const void* src, boo
                  "r"(valid ? 8 : 0));
 }
 
+// cp.async ordered after the preceding shared-memory reads of the same thread (the
+// store-then-reseed of a cube position: the "memory" clobber keeps the compiler from
+// moving the read of the old value past the copy that overwrites it)
+__device__ __forceinline__ void cp_async_8_after_read(void* dst, const void* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+
 __device__ __forceinline__ double flip_sign(double x, uint32_t mask_hi) {
     return __hiloint2double(__double2hiint(x) ^ (int)mask_hi, __double2loint(x));
 }
@@ -839,6 +846,7 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
             }
         }
     };
+    const bool full_cubes = P.qe[0] % BS == 0 && P.qe[1] % BS == 0 && P.qe[2] % BS == 0;
     int g = 0;
     for (int u = blockIdx.x; u < units; u += gridDim.x) {
         int o[3], len[3], qv[3];
@@ -846,8 +854,15 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
         const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
                               (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
         const int nvol = len[0] * len[1] * len[2];
-        named_bar_sync(1, 256);  // the previous unit's store from the cube is complete
-        seed(o, len, pbase, acc_s);  // lands while the first stages compute
+        // all cubes full: thread t owns positions (t & 15, t >> 4, *) in every unit, so the
+        // previous unit's store and this unit's seed were issued together at its end (no
+        // barrier); otherwise barrier, then seed
+        if (!full_cubes) {
+            named_bar_sync(1, 256);  // the previous unit's store from the cube is complete
+            seed(o, len, pbase, acc_s);  // lands while the first stages compute
+        } else if (u == (int)blockIdx.x) {
+            seed(o, len, pbase, acc_s);
+        }
         cp_async_commit();
         bool seeded = false;
 
@@ -902,7 +917,29 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_cons
             seeded = true;
         }
         named_bar_sync(1, 256);  // all flushes into this cube are done
-        if (len[0] == BS && len[1] == BS && len[2] == BS) {
+        if (full_cubes) {
+            // store this unit and seed the CTA's next unit, position by position (same owner)
+            const int q0 = tid & 15, q1 = tid >> 4;
+            double* dstg = P.t3 + pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)P.qe[1] * o[2]);
+            double* srcs = acc_s + q0 + CST * q1;
+            const int un = u + gridDim.x;
+            if (un < units) {
+                int on[3], lenn[3], qvn[3];
+                decode(un, on, lenn, qvn);
+                const int64_t pbn = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
+                                    (qvn[0] + (int64_t)P.qe[3] * (qvn[1] + (int64_t)P.qe[4] * qvn[2]));
+                const double* srcg = P.t3 + pbn + (on[0] + q0) + (int64_t)Q0 * ((on[1] + q1) + (int64_t)P.qe[1] * on[2]);
+#pragma unroll
+                for (int q2 = 0; q2 < BS; ++q2) {
+                    dstg[(int64_t)Q01 * q2] = srcs[CST * CST * q2];
+                    cp_async_8_after_read(srcs + CST * CST * q2, srcg + (int64_t)Q01 * q2);
+                }
+                cp_async_commit();
+            } else {
+#pragma unroll
+                for (int q2 = 0; q2 < BS; ++q2) dstg[(int64_t)Q01 * q2] = srcs[CST * CST * q2];
+            }
+        } else if (len[0] == BS && len[1] == BS && len[2] == BS) {
             const int q0 = tid & 15, q1 = tid >> 4;
             double* dstg = P.t3 + pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)P.qe[1] * o[2]);
             const double* srcs = acc_s + q0 + CST * q1;
@@ -1118,17 +1155,23 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
         const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
                               (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
         const int nvol = len[0] * len[1] * len[2];
-        named_bar_sync(1, NCT);  // the previous unit's store from the cube is complete
+        // Dense blocks: thread t owns cube positions i = t + NCT j in every unit, so the
+        // previous unit's store and this unit's seed (issued together at the end of the
+        // previous unit, below) need no barrier between them; only the CTA's first unit
+        // seeds here.  Ragged cubes: barrier, then seed.
         if (BC_EXP_NOSEED) {
         } else if (dense) {
-            const double* src = P.t3 + pbase;
+            if (u == (int)blockIdx.x) {
+                const double* src = P.t3 + pbase;
 #pragma unroll 6
-            for (int i = tid; i < BS * BS * BS; i += NCT) {
-                const int r = i / BS, q0 = i - r * BS;  // constant divisor: multiply-shift
-                const int q2 = r / BS, q1 = r - q2 * BS;
-                cp_async_8(acc_s + q0 + TG::C1 * q1 + TG::C2 * q2, src + i);
+                for (int i = tid; i < BS * BS * BS; i += NCT) {
+                    const int r = i / BS, q0 = i - r * BS;  // constant divisor: multiply-shift
+                    const int q2 = r / BS, q1 = r - q2 * BS;
+                    cp_async_8(acc_s + q0 + TG::C1 * q1 + TG::C2 * q2, src + i);
+                }
             }
         } else {
+            named_bar_sync(1, NCT);  // the previous unit's store from the cube is complete
             for (int i = tid; i < nvol; i += NCT) {
                 const int q0 = i % len[0], r = i / len[0];
                 const int q1 = r % len[1], q2 = r / len[1];
@@ -1234,13 +1277,20 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
         named_bar_sync(1, NCT);  // all flushes into this cube are done
         if (BC_EXP_NOSEED) {
         } else if (dense) {
+            // store this unit and seed the CTA's next unit position by position (same owner)
             double* dst = P.t3 + pbase;
+            const int un = u + gridDim.x;
+            const double* src = P.t3 + (int64_t)BS * BS * BS * (un < units ? un : u);
+            const bool next = un < units;
 #pragma unroll 6
             for (int i = tid; i < BS * BS * BS; i += NCT) {
                 const int r = i / BS, q0 = i - r * BS;
                 const int q2 = r / BS, q1 = r - q2 * BS;
-                dst[i] = acc_s[q0 + TG::C1 * q1 + TG::C2 * q2];
+                double* x = acc_s + q0 + TG::C1 * q1 + TG::C2 * q2;
+                dst[i] = *x;
+                if (next) cp_async_8_after_read(x, src + i);
             }
+            cp_async_commit();
         } else {
             for (int i = tid; i < nvol; i += NCT) {
                 const int q0 = i % len[0], r = i / len[0];
