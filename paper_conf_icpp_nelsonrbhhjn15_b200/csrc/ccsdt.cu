@@ -571,6 +571,9 @@ struct TmaMaps {
     CUtensorMap b[9];  // d1: t2_v (k,p4,p5,h1) | d2: v2_v (k,h3,p6,p5)
 };
 
+#ifndef BC_TC16_SINGLE_NS1
+#define BC_TC16_SINGLE_NS1 1
+#endif
 #ifndef BC_TC16_KC
 #define BC_TC16_KC 16
 #endif
@@ -757,11 +760,13 @@ __device__ __forceinline__ void tma_flush_class(double* acc_s, double (&c)[4][2]
     }
 }
 
-template <int FAM>
-__global__ void __launch_bounds__(TmaGeo::NT) ccsdt_tma_kernel(const __grid_constant__ CcsdtParams P,
-                                                               const __grid_constant__ TmaMaps M, int units) {
+// NSR: ring depth.  Single-variant launches (one stage per unit at tile 16) use NSR = 1
+// and 3 CTAs/SM: more units (t3 seeds) in flight for the HBM-bound case.
+template <int FAM, int NSR = TmaGeo::NS, int MINB = 2>
+__global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __grid_constant__ CcsdtParams P,
+                                                                     const __grid_constant__ TmaMaps M, int units) {
     using TG = TmaGeo;
-    constexpr int BS = TG::BS, KC = TG::KC, NS = TG::NS, CST = TG::CST;
+    constexpr int BS = TG::BS, KC = TG::KC, NS = NSR, CST = TG::CST;
     extern __shared__ unsigned char smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
     const uint32_t base = (raw + 1023) & ~1023u;
@@ -1022,18 +1027,23 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
         }
         if (!ok) return 1;
     }
-    static int occ = 0;
-    if (occ == 0) {
-        cudaFuncSetAttribute(ccsdt_tma_kernel<FAM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TmaGeo::SMEM);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_tma_kernel<FAM>, TmaGeo::NT, TmaGeo::SMEM);
-        if (occ < 1) occ = 1;
-    }
     const int64_t units = (int64_t)P.ncube[0] * P.ncube[1] * P.ncube[2] * P.qe[3] * P.qe[4] * P.qe[5];
     if (units == 0) return BC_OK;
-    const int64_t cap = (int64_t)num_sms() * occ;
-    const int grid = (int)(units < cap ? units : cap);
-    ccsdt_tma_kernel<FAM><<<grid, TmaGeo::NT, TmaGeo::SMEM, s>>>(P, M, (int)units);
-    return launch_status();
+    auto go = [&](auto kern, size_t smem, int* occ) {
+        if (*occ == 0) {
+            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, kern, TmaGeo::NT, smem);
+            if (*occ < 1) *occ = 1;
+        }
+        const int64_t cap = (int64_t)num_sms() * *occ;
+        const int grid = (int)(units < cap ? units : cap);
+        kern<<<grid, TmaGeo::NT, smem, s>>>(P, M, (int)units);
+        return launch_status();
+    };
+    const size_t smem1 = 1024 + (size_t)TmaGeo::STAGE_BYTES + TmaGeo::ACC * 8 + 2 * 8;
+    static int occ = 0, occ1 = 0;
+    if (P.nentry == 1 && BC_TC16_SINGLE_NS1) return go(ccsdt_tma_kernel<FAM, 1, 3>, smem1, &occ1);
+    return go(ccsdt_tma_kernel<FAM>, TmaGeo::SMEM, &occ);
 }
 
 // ==================================================================================
