@@ -1624,6 +1624,308 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
     return run_check_finalize(grid, ws, s);
 }
 
+// ==================================================================================
+// s1 streaming path (single or fused variants sharing one t3 geometry).  s1 has no
+// contracted index: t3[sigma_v] += s_v t1[p4,h1] v2[h3,h2,p6,p5] is a rank-1 update per
+// particle plane, so the kernel is a pure t3 read-modify-write stream (AI 2 flop / 16 B per
+// variant).  A CTA owns whole particle planes (the hole volume of a plane is contiguous in
+// t3 for every storage order, since the holes are the three fastest positions): it stages
+// the plane's per-entry factors in shared memory — Vs_e[h2][h3] = s_e v2_e[h3,h2,p6,p5]
+// (row stride H3+1: conflict-free whichever hole name runs along the lanes) and
+// Ts_e[h1] = t1_e[p4,h1] — then streams the plane's t3 values with all of a thread's
+// loads in flight at once.  Per element and entry: 2 shared loads and one FMA; the hole
+// names of an element are linear forms of its storage coordinates, one per class.
+// ==================================================================================
+constexpr int S1S_NT = 256, S1S_U = 8;  // threads, t3 values in flight per thread
+
+__global__ void __launch_bounds__(S1S_NT) ccsdt_s1_stream_kernel(const __grid_constant__ CcsdtParams P,
+                                                                 int nplanes) {
+    extern __shared__ __align__(16) double s1sm[];
+    const int H1 = P.ext[N_H1], H2 = P.ext[N_H2], H3 = P.ext[N_H3];
+    const int P4 = P.ext[N_P4], P6 = P.ext[N_P6];
+    const int VS = H2 * (H3 + 1), ES = VS + H1;   // per entry: Vs [h2][h3] (row stride H3+1), Ts [h1]
+    const int BUFD = P.nentry * ES;               // one plane's factors (2 buffers)
+    const int Q0 = P.qe[0], Q1 = P.qe[1], Q2 = P.qe[2];
+    const int nh = Q0 * Q1 * Q2;
+    const int tid = threadIdx.x;
+    // entries are grouped by class (run_ccsdt): slot (c, m) = entry cb[c] + m, m < cnt[c]
+    int n0 = 0, n1 = 0, n2 = 0;
+    for (int e = 0; e < P.nentry; ++e) {
+        const int c = P.ecls[e];
+        n0 += c == 0;
+        n1 += c == 1;
+        n2 += c == 2;
+    }
+    const int cb[3] = {0, n0, n0 + n1}, cnt[3] = {n0, n1, n2};
+    uint32_t sm_[3][3];
+    int av[3][3], at[3][3];
+#pragma unroll
+    for (int c = 0; c < 3; ++c) {
+#pragma unroll
+        for (int m = 0; m < 3; ++m) sm_[c][m] = (m < cnt[c]) ? P.smask[cb[c] + m] : 0u;
+#pragma unroll
+        for (int q = 0; q < 3; ++q) {
+            const bool ok = c < P.ncls;
+            at[c][q] = (ok && P.hpos[c][0] == q) ? 1 : 0;                                            // h1
+            av[c][q] = (ok && P.hpos[c][1] == q) ? H3 + 1 : ((ok && P.hpos[c][2] == q) ? 1 : 0);  // h2, h3
+        }
+    }
+    // stage plane j's factors into buffer b (cp.async; signs are applied at use)
+    auto stage = [&](int plane, int b) {
+        const int qv0 = plane % P.qe[3], qv1 = (plane / P.qe[3]) % P.qe[4], qv2 = plane / (P.qe[3] * P.qe[4]);
+        auto pick = [&](int pos) { return pos == 3 ? qv0 : (pos == 4 ? qv1 : qv2); };
+        double* buf = s1sm + b * BUFD;
+        for (int e = 0; e < P.nentry; ++e) {
+            const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
+            const double* v2 = P.opB[e] + (int64_t)H3 * H2 * (p6 + (int64_t)P6 * p5);
+            for (int i = tid; i < H2 * H3; i += S1S_NT) {
+                const int h2 = i / H3, h3 = i - h2 * H3;
+                cp_async_8(buf + e * ES + h2 * (H3 + 1) + h3, v2 + i);
+            }
+            const double* t1 = P.opA[e] + p4;
+            for (int h1 = tid; h1 < H1; h1 += S1S_NT) cp_async_8(buf + e * ES + VS + h1, t1 + (int64_t)P4 * h1);
+        }
+    };
+    // this thread's storage coordinates at i = tid and the step for i += S1S_NT
+    const int iq0 = tid % Q0, iq1 = (tid / Q0) % Q1, iq2 = tid / (Q0 * Q1);
+    const int d0 = S1S_NT % Q0, d1 = (S1S_NT / Q0) % Q1, d2 = S1S_NT / (Q0 * Q1);
+    int it = 0;
+    if ((int)blockIdx.x < nplanes) stage(blockIdx.x, 0);
+    cp_async_commit();
+    for (int plane = blockIdx.x; plane < nplanes; plane += gridDim.x, ++it) {
+        cp_async_wait_all();
+        __syncthreads();  // this plane's factors landed; the other buffer is free
+        if (plane + (int)gridDim.x < nplanes) stage(plane + gridDim.x, (it + 1) & 1);
+        cp_async_commit();
+        const double* buf = s1sm + (it & 1) * BUFD;
+        double* t3p = P.t3 + (int64_t)nh * plane;
+        int q0 = iq0, q1 = iq1, q2 = iq2;
+        for (int i0 = 0; i0 < nh; i0 += S1S_NT * S1S_U) {
+            double x[S1S_U];
+#pragma unroll
+            for (int u = 0; u < S1S_U; ++u) {
+                const int i = i0 + u * S1S_NT + tid;
+                x[u] = (i < nh) ? __ldcs(t3p + i) : 0.0;
+            }
+#pragma unroll
+            for (int u = 0; u < S1S_U; ++u) {
+                const int i = i0 + u * S1S_NT + tid;
+                if (i < nh) {
+                    double acc = x[u];
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) {
+                        const int vo = q0 * av[c][0] + q1 * av[c][1] + q2 * av[c][2];
+                        const int to = VS + q0 * at[c][0] + q1 * at[c][1] + q2 * at[c][2];
+#pragma unroll
+                        for (int m = 0; m < 3; ++m)
+                            if (m < cnt[c]) {
+                                const double* eb = buf + (cb[c] + m) * ES;
+                                acc = fma(flip_sign(eb[to], sm_[c][m]), eb[vo], acc);
+                            }
+                    }
+                    __stcs(t3p + i, acc);
+                }
+                // advance (q0, q1, q2) by S1S_NT elements
+                q0 += d0;
+                const int c0 = q0 >= Q0;
+                q0 -= c0 ? Q0 : 0;
+                q1 += d1 + c0;
+                const int c1 = q1 >= Q1;
+                q1 -= c1 ? Q1 : 0;
+                q2 += d2 + c1;
+            }
+        }
+    }
+}
+
+static int launch_ccsdt_s1_stream(const CcsdtParams& P, cudaStream_t s) {
+    const size_t smem = 2 * ((size_t)P.nentry * (P.ext[N_H2] * (P.ext[N_H3] + 1) + P.ext[N_H1])) * 8;
+    if (smem > 200 * 1024) return 1;
+    const int nplanes = P.qe[3] * P.qe[4] * P.qe[5];
+    if (nplanes == 0 || P.qe[0] * P.qe[1] * P.qe[2] == 0) return BC_OK;
+    static size_t last_smem = 0;
+    static int occ = 0;
+    if (smem != last_smem) {
+        cudaFuncSetAttribute(ccsdt_s1_stream_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_s1_stream_kernel, S1S_NT, smem);
+        if (occ < 1) occ = 1;
+        last_smem = smem;
+    }
+    const int64_t cap = (int64_t)num_sms() * occ;
+    const int grid = (int)(nplanes < cap ? nplanes : cap);
+    ccsdt_s1_stream_kernel<<<grid, S1S_NT, smem, s>>>(P, nplanes);
+    return launch_status();
+}
+
+// ==================================================================================
+// Single-variant d1/d2 streaming path (hole extents 16^3, one variant per call: the
+// HBM-bound configs 3/4 per-variant rows).  One variant touches each t3 value once, so
+// the kernel streams t3 planes (the 16^3 hole volume of one particle triple is 32 KB
+// contiguous in every storage order) through registers: the thread's 16 t3 values are
+// the initial values of its 4 x 4 DFMA accumulator tile, t3 += sum_k A B is accumulated in
+// place and stored — no shared-memory cube, no flush.  The next plane's t3 values and B
+// slice are in flight while the current plane computes.
+//   GEMM per plane: X[(f, x), y] = sum_k A[k][f][x] B[k][y]
+//     d1: f = h2, x = h3, y = h1;  A = s v2[h3,h2,p6,k] (per p6),  B = t2[k,p4,p5,h1]
+//     d2: f = h1, x = h2, y = h3;  A = s t2[k,p4,h1,h2] (per p4),  B = v2[k,h3,p6,p5]
+// Storage position 0 is always x or y (d1: h3 or h1; d2: h3 or h2), so a thread's 4 x 4
+// tile is 4 rows of 4 contiguous t3 values (two 16-byte accesses each) and 4 lanes cover a
+// 128-byte run.  Planes are visited with the A name slowest, so A (sign folded) is staged
+// once per CTA or twice.
+// ==================================================================================
+constexpr int SV_NT = 256, SV_RS = 18, SV_PS = 16 * SV_RS + 2;  // A row / k-plane strides (doubles)
+
+__device__ __forceinline__ double2 ld_cs2(const double* p) { return __ldcs(reinterpret_cast<const double2*>(p)); }
+__device__ __forceinline__ void st_cs2(double* p, double a, double b) {
+    __stcs(reinterpret_cast<double2*>(p), make_double2(a, b));
+}
+
+template <int FAM>
+__global__ void __launch_bounds__(SV_NT, 2) ccsdt_sv16_kernel(const __grid_constant__ CcsdtParams P, int nplanes) {
+    extern __shared__ __align__(16) double svsm[];
+    const int K = P.ext[N_K];
+    double* As = svsm;                 // [k][f][x] (row stride SV_RS, k-plane stride SV_PS)
+    double* Bs = As + K * SV_PS;       // 2 buffers of [k][y]
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int* hp = P.hpos[0];         // storage positions of h1, h2, h3
+    const int posX = (FAM == FAM_D1) ? hp[2] : hp[1];
+    const int posY = (FAM == FAM_D1) ? hp[0] : hp[2];
+    const int posF = (FAM == FAM_D1) ? hp[1] : hp[0];
+    const bool xfast = posX == 0;      // else posY == 0
+    const int bq = lane & 3, bo = (lane >> 2) & 3;
+    const int bx = xfast ? bq : bo, by = xfast ? bo : bq;
+    const int f = 2 * warp + (lane >> 4);
+    const int sX = 1 << (4 * posX), sY = 1 << (4 * posY), sF = 1 << (4 * posF);
+    // the tile's 4 rows of 4 contiguous values: row r -> offset, element c contiguous
+    const int rstride = xfast ? sY : sX;
+    const int tbase = 4 * bx * sX + 4 * by * sY + f * sF;
+    // particle names: A name a (d1 p6, d2 p4) slowest, then o1, o2
+    const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6];
+    const int PO1 = (FAM == FAM_D1) ? P5 : P6, PO2 = (FAM == FAM_D1) ? P4 : P5;
+    auto qstride = [&](int pos) {
+        return pos == 3 ? 4096LL : (pos == 4 ? 4096LL * P.qe[3] : 4096LL * P.qe[3] * P.qe[4]);
+    };
+    const int64_t sp4 = qstride(P.ppos[0][0]), sp5 = qstride(P.ppos[0][1]), sp6 = qstride(P.ppos[0][2]);
+    const double sg = P.sign[0];
+    const double* __restrict__ opA = P.opA[0];  // t2
+    const double* __restrict__ opB = P.opB[0];  // v2
+
+    const int lo = (int)((int64_t)nplanes * blockIdx.x / gridDim.x);
+    const int hi = (int)((int64_t)nplanes * (blockIdx.x + 1) / gridDim.x);
+    auto names = [&](int j, int& a, int& o1, int& o2) {
+        a = j / (PO1 * PO2);
+        const int r = j - a * (PO1 * PO2);
+        o1 = r / PO2;
+        o2 = r - o1 * PO2;
+    };
+    auto plane_ptr = [&](int j) {
+        int a, o1, o2;
+        names(j, a, o1, o2);
+        const int p4 = (FAM == FAM_D1) ? o2 : a, p5 = (FAM == FAM_D1) ? o1 : o2, p6 = (FAM == FAM_D1) ? a : o1;
+        return P.t3 + p4 * sp4 + p5 * sp5 + p6 * sp6 + tbase;
+    };
+    auto issue_B = [&](int j, double* dst) {  // B[k][y], 16 K values
+        int a, o1, o2;
+        names(j, a, o1, o2);
+        const double* src = (FAM == FAM_D1) ? opA + (int64_t)K * (o2 + (int64_t)P4 * o1)       // t2[k,p4,p5,h1]
+                                            : opB + (int64_t)K * 16 * (o1 + (int64_t)P6 * o2);  // v2[k,h3,p6,p5]
+        const int stride_y = (FAM == FAM_D1) ? K * P4 * P5 : K;
+        for (int i = tid; i < 16 * K; i += SV_NT) {
+            const int y = i / K, k = i - y * K;
+            cp_async_8(dst + k * 16 + y, src + (int64_t)stride_y * y + k);
+        }
+    };
+    auto load_tile = [&](const double* p, double (&x)[4][4]) {
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            const double2 u = ld_cs2(p + r * rstride), w = ld_cs2(p + r * rstride + 2);
+            x[r][0] = u.x; x[r][1] = u.y; x[r][2] = w.x; x[r][3] = w.y;
+        }
+    };
+    if (lo >= hi) return;
+    double x[4][4];  // [row][c]: xfast -> (y = row, x = c), else (x = row, y = c)
+    load_tile(plane_ptr(lo), x);
+    issue_B(lo, Bs);
+    cp_async_commit();
+    int curA = -1;
+    for (int j = lo; j < hi; ++j) {
+        int a, o1, o2;
+        names(j, a, o1, o2);
+        if (a != curA) {
+            __syncthreads();  // every thread is done with the previous A
+            if (FAM == FAM_D1) {  // As[k][h2][h3] = s v2[h3,h2,p6,k]
+                const double* src = opB + 256LL * a;
+                for (int i = tid; i < 256 * K; i += SV_NT) {
+                    const int k = i >> 8, r = i & 255;
+                    As[k * SV_PS + (r >> 4) * SV_RS + (r & 15)] = sg * __ldg(src + (int64_t)256 * P6 * k + r);
+                }
+            } else {  // As[k][h1][h2] = s t2[k,p4,h1,h2]
+                const double* src = opA + (int64_t)K * a;
+                for (int i = tid; i < 256 * K; i += SV_NT) {
+                    const int r = i / K, k = i - r * K;  // r = h1 + 16 h2
+                    As[k * SV_PS + (r & 15) * SV_RS + (r >> 4)] = sg * __ldg(src + (int64_t)K * P4 * r + k);
+                }
+            }
+            curA = a;
+        }
+        cp_async_wait_all();
+        __syncthreads();  // B(j) landed, A staged, the other B buffer is free
+        const double* Bc = Bs + ((j - lo) & 1) * 16 * K;
+        if (j + 1 < hi) issue_B(j + 1, Bs + ((j + 1 - lo) & 1) * 16 * K);
+        cp_async_commit();
+        double acc[4][4];
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) acc[r][c] = x[r][c];
+        double* tp = plane_ptr(j);
+        if (j + 1 < hi) load_tile(plane_ptr(j + 1), x);
+        const double* Ap = As + f * SV_RS + 4 * bx;
+        const double* Bp = Bc + 4 * by;
+#pragma unroll 4
+        for (int k = 0; k < K; ++k) {
+            const double2 a01 = *reinterpret_cast<const double2*>(Ap + k * SV_PS);
+            const double2 a23 = *reinterpret_cast<const double2*>(Ap + k * SV_PS + 2);
+            const double2 b01 = *reinterpret_cast<const double2*>(Bp + k * 16);
+            const double2 b23 = *reinterpret_cast<const double2*>(Bp + k * 16 + 2);
+            const double av[4] = {a01.x, a01.y, a23.x, a23.y}, bv[4] = {b01.x, b01.y, b23.x, b23.y};
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+#pragma unroll
+                for (int jj = 0; jj < 4; ++jj) {
+                    // xfast: row = y (jj), element = x (i); else row = x (i), element = y (jj)
+                    double& t = xfast ? acc[jj][i] : acc[i][jj];
+                    t = fma(av[i], bv[jj], t);
+                }
+        }
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            st_cs2(tp + r * rstride, acc[r][0], acc[r][1]);
+            st_cs2(tp + r * rstride + 2, acc[r][2], acc[r][3]);
+        }
+    }
+}
+
+template <int FAM>
+static int launch_ccsdt_sv16(const CcsdtParams& P, cudaStream_t s) {
+    const int K = P.ext[N_K];
+    const size_t smem = ((size_t)K * SV_PS + 2 * 16 * (size_t)K) * 8;
+    const int nplanes = P.qe[3] * P.qe[4] * P.qe[5];
+    if (nplanes == 0) return BC_OK;
+    static size_t last_smem = 0;
+    static int occ = 0;
+    if (smem != last_smem) {
+        cudaFuncSetAttribute(ccsdt_sv16_kernel<FAM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_sv16_kernel<FAM>, SV_NT, smem);
+        if (occ < 1) occ = 1;
+        last_smem = smem;
+    }
+    const int64_t cap = (int64_t)num_sms() * occ;
+    const int grid = (int)(nplanes < cap ? nplanes : cap);
+    ccsdt_sv16_kernel<FAM><<<grid, SV_NT, smem, s>>>(P, nplanes);
+    return launch_status();
+}
+
 // ------------------------------------------------------------------------------------ host
 static int choose_bs(const int* qe) {
     // smallest padded volume over the three hole positions; ties -> larger cube
@@ -1686,6 +1988,14 @@ int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const
     }
     P.nentry = n;
     P.ncls = ncls;
+    if (fam == FAM_S1 && getenv("BC_NO_S1STREAM") == nullptr) {
+        const int st = launch_ccsdt_s1_stream(P, s);
+        if (st != 1) return st;  // 1: factors exceed shared memory (cube kernel below)
+    }
+    // one d1/d2 variant on 16^3 hole cubes: t3 streamed through registers (HBM-bound)
+    if (n == 1 && fam != FAM_S1 && ext7[N_H1] == 16 && ext7[N_H2] == 16 && ext7[N_H3] == 16 && ext7[N_K] <= 32 &&
+        getenv("BC_NO_SV16") == nullptr)
+        return fam == FAM_D1 ? launch_ccsdt_sv16<FAM_D1>(P, s) : launch_ccsdt_sv16<FAM_D2>(P, s);
     // tensor-core path: 16-cubes with 16-byte-aligned operand rows (even k, even h3 for d1).
     // It also takes hole extents the 16-cube does not divide (e.g. tile 24 = 16 + 8, ragged
     // cubes zero-filled by TMA): measured 2x faster than the 12-cube DFMA kernel at tile 24.

@@ -18,6 +18,15 @@
 #ifndef BC_NUNROLL
 #define BC_NUNROLL 1
 #endif
+// warp-chunked line assignment (no duplicate tail lines; measured: p=12 local_grad3
+// 0.686 -> 0.726, p=9 0.79 -> 0.86 of HBM) and the software-pipelined n loop (measured
+// slower: +50 registers, 0.73 -> 0.58 at p=12; kept as an option)
+#ifndef BC_WCHUNK
+#define BC_WCHUNK 1
+#endif
+#ifndef BC_SWP
+#define BC_SWP 0
+#endif
 
 namespace bc {
 
@@ -40,23 +49,26 @@ struct Geo {
     static constexpr bool VEC_ROWS = (sizeof(T) == 8) && (RS % 2 == 0);
 };
 
-// Stage `ne` elements (contiguous in global from `src`) into padded smem `dst`.
+// Stage `ne` elements (contiguous in global from `src`) into padded smem at `dst` (16-byte
+// aligned, VEC elements of slack at the end).  Returns where element 0 landed: for an
+// unpadded fp64 group that starts 8 bytes past a 16-byte boundary (odd E x odd P1) the copy
+// starts one value early, so element 0 sits at dst + 1 and every copy stays 16 bytes wide.
 template <int P1, int NA, typename T, int NT>
-__device__ __forceinline__ void load_group_async(T* __restrict__ dst, const T* __restrict__ src,
-                                                 int ne) {
+__device__ __forceinline__ T* load_group_async(T* __restrict__ dst, const T* __restrict__ src, int ne) {
     using G = Geo<P1, NA, T>;
     const int total = ne * G::NPTS;
     if constexpr (!G::PADDED) {
-        // smem layout == global layout: 16-byte chunks when aligned
+        // smem layout == global layout: 16-byte chunks
         constexpr int V = 16 / sizeof(T);
-        const bool aligned = ((reinterpret_cast<uintptr_t>(src) & 15) == 0);
-        if (aligned) {
-            const int nvec = total / V;
-            for (int i = threadIdx.x; i < nvec; i += NT) cp_async_16(dst + i * V, src + i * V);
-            for (int i = nvec * V + threadIdx.x; i < total; i += NT) cp_async_elem(dst + i, src + i);
-        } else {
-            for (int i = threadIdx.x; i < total; i += NT) cp_async_elem(dst + i, src + i);
+        const int lead = (int)((reinterpret_cast<uintptr_t>(src) & 15) / sizeof(T));
+        if (sizeof(T) == 8 || lead == 0) {
+            const T* s0 = src - lead;
+            const int tot = total + lead, nvec = tot / V;
+            for (int i = threadIdx.x; i < nvec; i += NT) cp_async_16(dst + i * V, s0 + i * V);
+            for (int i = nvec * V + threadIdx.x; i < tot; i += NT) cp_async_elem(dst + i, s0 + i);
+            return dst + lead;
         }
+        for (int i = threadIdx.x; i < total; i += NT) cp_async_elem(dst + i, src + i);
     } else {
         for (int f = threadIdx.x; f < total; f += NT) {
             const int e = f / G::NPTS;
@@ -66,6 +78,7 @@ __device__ __forceinline__ void load_group_async(T* __restrict__ dst, const T* _
             cp_async_elem(dst + e * G::ES + row * G::RS + c, src + f);
         }
     }
+    return dst;
 }
 
 // smem offset of global point f (element-relative flattened (e, a, b, c))
@@ -129,8 +142,15 @@ struct Line {
 // 16-byte broadcast operator load feeds 2R FMAs and there are P1*R independent FMA
 // chains per thread.  All reads of a line precede the writes of that line and every
 // line is read by exactly one thread, so `out` may overwrite the line in place.
+template <int P1, int NA, int AXIS, int R, int NT, bool SWP, typename T, typename Out>
+__device__ __forceinline__ void apply_lines_w(const T* in, const T* opT, int nlines, Out out);
+
 template <int P1, int NA, int AXIS, int R, int NT, typename T, typename Out, int UNR = BC_NUNROLL>
 __device__ __forceinline__ void apply_lines(const T* in, const T* opT, int nlines, Out out) {
+    if constexpr (BC_WCHUNK && UNR == 1) {
+        apply_lines_w<P1, NA, AXIS, R, NT, (bool)BC_SWP>(in, opT, nlines, out);
+        return;
+    }
     using G = Geo<P1, NA, T>;
     using LN = Line<P1, NA, AXIS, T>;
     using P2 = typename Pair<T>::type;
@@ -175,6 +195,97 @@ __device__ __forceinline__ void apply_lines(const T* in, const T* opT, int nline
 #pragma unroll
                 for (int k = 0; k < P1; ++k) out(L0 + r * NT, base[r], k, acc[k][r]);
             }
+    }
+}
+
+// One warp chunk of apply_lines: lane `lane` owns lines L0 + r*32 (r < RR), lines >= nlines
+// are computed on the chunk's first line (always valid) and not stored.  SWP: the operands of step n+1 are loaded
+// while step n's FMAs run (two register sets, ping-pong), hiding the shared-memory latency
+// that otherwise stalls every step's first FMA.
+template <int P1, int NA, int AXIS, int RR, bool SWP, typename T, typename Out>
+__device__ __forceinline__ void lines_chunk(const T* in, const T* opT, int L0, int nlines, Out& out) {
+    using G = Geo<P1, NA, T>;
+    using LN = Line<P1, NA, AXIS, T>;
+    using P2 = typename Pair<T>::type;
+    constexpr int KP = P1 / 2;
+    int base[RR];
+#pragma unroll
+    for (int r = 0; r < RR; ++r) {
+        const int L = L0 + r * 32;
+        base[r] = LN::base(L < nlines ? L : (L0 & ~31));
+    }
+    T acc[P1][RR];
+#pragma unroll
+    for (int k = 0; k < P1; ++k)
+#pragma unroll
+        for (int r = 0; r < RR; ++r) acc[k][r] = T(0);
+    auto fmas = [&](const T (&x)[RR], const P2 (&o)[KP], T oz) {
+#pragma unroll
+        for (int k2 = 0; k2 < KP; ++k2)
+#pragma unroll
+            for (int r = 0; r < RR; ++r) {
+                acc[2 * k2][r] = fma(o[k2].x, x[r], acc[2 * k2][r]);
+                acc[2 * k2 + 1][r] = fma(o[k2].y, x[r], acc[2 * k2 + 1][r]);
+            }
+        if constexpr (P1 & 1) {
+#pragma unroll
+            for (int r = 0; r < RR; ++r) acc[P1 - 1][r] = fma(oz, x[r], acc[P1 - 1][r]);
+        }
+    };
+    auto ld = [&](int n, T (&x)[RR], P2 (&o)[KP], T& oz) {
+#pragma unroll
+        for (int r = 0; r < RR; ++r) x[r] = in[base[r] + n * LN::STRIDE];
+        const T* orow = opT + n * G::OS;
+#pragma unroll
+        for (int k2 = 0; k2 < KP; ++k2) o[k2] = reinterpret_cast<const P2*>(orow)[k2];
+        if constexpr (P1 & 1) oz = orow[P1 - 1];
+    };
+    if constexpr (SWP) {
+        T xa[RR], xb[RR], za = T(0), zb = T(0);
+        P2 oa[KP], ob[KP];
+        ld(0, xa, oa, za);
+#pragma unroll 1
+        for (int n = 0; n + 1 < P1; n += 2) {
+            ld(n + 1, xb, ob, zb);
+            fmas(xa, oa, za);
+            if (n + 2 < P1) ld(n + 2, xa, oa, za);
+            fmas(xb, ob, zb);
+        }
+        if constexpr (P1 & 1) fmas(xa, oa, za);
+    } else {
+#pragma unroll 1
+        for (int n = 0; n < P1; ++n) {
+            T x[RR], z = T(0);
+            P2 o[KP];
+            ld(n, x, o, z);
+            fmas(x, o, z);
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < RR; ++r)
+        if (L0 + r * 32 < nlines) {
+#pragma unroll
+            for (int k = 0; k < P1; ++k) out(L0 + r * 32, base[r], k, acc[k][r]);
+        }
+}
+
+// Warp-chunked form of apply_lines (same arithmetic, same ascending-n sums): lines are cut
+// into chunks of 32*R (lane-interleaved, so every strided line read stays conflict-free);
+// chunks go round-robin to the warps and the ragged last chunk runs with
+// RR = ceil(rest/32) <= R lines per lane, so no warp computes duplicate lines.
+template <int P1, int NA, int AXIS, int R, int NT, bool SWP, typename T, typename Out>
+__device__ __forceinline__ void apply_lines_w(const T* in, const T* opT, int nlines, Out out) {
+    constexpr int NW = NT / 32, CH = 32 * R;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int nfull = nlines / CH;
+    for (int c = warp; c < nfull; c += NW) lines_chunk<P1, NA, AXIS, R, SWP>(in, opT, c * CH + lane, nlines, out);
+    const int rest = nlines - nfull * CH;
+    if (rest > 0 && warp == nfull % NW) {
+        const int L0 = nfull * CH + lane, rr = (rest + 31) >> 5;
+        if constexpr (R >= 4) if (rr == 4) { lines_chunk<P1, NA, AXIS, 4, SWP>(in, opT, L0, nlines, out); return; }
+        if constexpr (R >= 3) if (rr == 3) { lines_chunk<P1, NA, AXIS, (R >= 3 ? 3 : 1), SWP>(in, opT, L0, nlines, out); return; }
+        if constexpr (R >= 2) if (rr == 2) { lines_chunk<P1, NA, AXIS, (R >= 2 ? 2 : 1), SWP>(in, opT, L0, nlines, out); return; }
+        lines_chunk<P1, NA, AXIS, 1, SWP>(in, opT, L0, nlines, out);
     }
 }
 
@@ -229,6 +340,9 @@ enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
 #ifndef BC_BIG_PF
 #define BC_BIG_PF 0
 #endif
+#ifndef BC_E13
+#define BC_E13 3
+#endif
 #ifndef BC_SF2_UNROLL
 #define BC_SF2_UNROLL 1
 #endif
@@ -240,6 +354,9 @@ struct SpecTable {
     static constexpr int R = BIG ? (SF3LG3 ? (MID ? 3 : BC_BIG_R) : (KIND == K_SF2 ? 3 : 2)) : 2;
     static constexpr int BUF_KB = BIG ? (SF3LG3 ? (MID ? 36 : BC_BIG_KB) : 18) : (KIND == K_LG3 ? 36 : 18);
     static constexpr bool PREFETCH = !(BIG && SF3LG3) || BC_BIG_PF;
+    // forced elements per group (0: derived from BUF_KB): P1 = 13: 3 x 169 = 507 lines on
+    // 128 threads x R = 4 (1% idle lanes instead of 12% with E = 2 on 96 threads)
+    static constexpr int EF = (SF3LG3 && P1 == 13) ? BC_E13 : 0;
     // unroll of the contracted-index loop: sumfact2d fully (its two stages fit the registers)
     static constexpr int UNROLL = (KIND == K_SF2 && BC_SF2_UNROLL && P1 >= 9) ? P1 : BC_NUNROLL;
 };
@@ -252,13 +369,15 @@ struct Cfg {
     static constexpr int NBUF = NBUF_FIELDS + (PREFETCH ? 1 : 0);
     static constexpr int BUF_BYTES = TB::BUF_KB * 1024;  // target bytes per element-group buffer
     static constexpr int E0 = BUF_BYTES / (G::ES * (int)sizeof(T));
-    static constexpr int E = E0 < 2 ? 1 : (E0 & ~1);  // even: groups of odd-P1 elements stay 16B-aligned
+    // even by default; a measured table entry may force E (odd E x odd P1 groups start 8 bytes
+    // off a 16-byte boundary, handled by load_group_async)
+    static constexpr int E = TB::EF ? TB::EF : (E0 < 2 ? 1 : (E0 & ~1));
     static constexpr int R = TB::R;
     static constexpr int LINES = E * NA * P1;  // lines per axis per group (E * NPTS / P1)
     static constexpr int NT0 = ((LINES + R - 1) / R + 31) / 32 * 32;
     static constexpr int NT = NT0 < 64 ? 64 : (NT0 > 512 ? 512 : NT0);
     static constexpr int VEC = 16 / (int)sizeof(T);
-    static constexpr int BUF = (E * G::ES + VEC - 1) / VEC * VEC;
+    static constexpr int BUF = (E * G::ES + VEC - 1) / VEC * VEC + VEC;  // + slack for a shifted group
     static constexpr size_t SMEM = (size_t)NBUF * BUF * sizeof(T) + 2 * op_elems<P1, T>() * sizeof(T);
 };
 
@@ -283,30 +402,32 @@ __device__ __forceinline__ void group_loop(int64_t N, const T* __restrict__ src,
     const int64_t ngroups = (N + E - 1) / E;
     if constexpr (PREFETCH) {
         int64_t g = blockIdx.x;
-        if (g < ngroups) load_group_async<P1, NA, T, NT>(buf0, src + g * E * G::NPTS, imin64(E, N - g * E));
+        T* in = buf0;
+        if (g < ngroups) in = load_group_async<P1, NA, T, NT>(buf0, src + g * E * G::NPTS, imin64(E, N - g * E));
         cp_async_commit();
         int cur = 0;
         for (; g < ngroups; g += gridDim.x) {
             const int64_t e0 = g * E;
             cp_async_wait_all();
             __syncthreads();  // group g landed; everyone is done with the other buffer
-            T* in = buf0 + cur * BUF;
             const int64_t gn = g + gridDim.x;
+            T* next = buf0 + (cur ^ 1) * BUF;
             if (gn < ngroups)
-                load_group_async<P1, NA, T, NT>(buf0 + (cur ^ 1) * BUF, src + gn * E * G::NPTS, imin64(E, N - gn * E));
+                next = load_group_async<P1, NA, T, NT>(next, src + gn * E * G::NPTS, imin64(E, N - gn * E));
             cp_async_commit();
             body(in, e0, imin64(E, N - e0));
+            in = next;
             cur ^= 1;
         }
     } else {
         for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
             const int64_t e0 = g * E;
             __syncthreads();  // everyone is done with the buffer
-            load_group_async<P1, NA, T, NT>(buf0, src + e0 * G::NPTS, imin64(E, N - e0));
+            T* in = load_group_async<P1, NA, T, NT>(buf0, src + e0 * G::NPTS, imin64(E, N - e0));
             cp_async_commit();
             cp_async_wait_all();
             __syncthreads();
-            body(buf0, e0, imin64(E, N - e0));
+            body(in, e0, imin64(E, N - e0));
         }
     }
 }
@@ -459,9 +580,9 @@ local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __re
     constexpr int E = CF::E, NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* opT = reinterpret_cast<T*>(smem_raw);
-    T* bR = opT + 2 * op_elems<P1, T>();
-    T* bS = bR + CF::BUF;
-    T* bT = bS + CF::BUF;
+    T* bR0 = opT + 2 * op_elems<P1, T>();
+    T* bS0 = bR0 + CF::BUF;
+    T* bT0 = bS0 + CF::BUF;
     load_op<P1, T, NT, true>(opT, D);
     const int64_t ngroups = (N + E - 1) / E;
     for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
@@ -470,9 +591,9 @@ local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __re
         const int nlines = ne * P1 * P1;
         const int64_t gbase = e0 * G::NPTS;
         __syncthreads();  // previous group fully consumed
-        load_group_async<P1, P1, T, NT>(bR, ur + gbase, ne);
-        load_group_async<P1, P1, T, NT>(bS, us + gbase, ne);
-        load_group_async<P1, P1, T, NT>(bT, ut + gbase, ne);
+        T* bR = load_group_async<P1, P1, T, NT>(bR0, ur + gbase, ne);
+        T* bS = load_group_async<P1, P1, T, NT>(bS0, us + gbase, ne);
+        T* bT = load_group_async<P1, P1, T, NT>(bT0, ut + gbase, ne);
         cp_async_commit();
         cp_async_wait_all();
         __syncthreads();
@@ -513,8 +634,8 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* opD = reinterpret_cast<T*>(smem_raw);
     T* opT = opD + op_elems<P1, T>();
-    T* bR = opT + op_elems<P1, T>();  // holds U, then ur / wr
-    T* bS = bR + CF::BUF;
+    T* bR0 = opT + op_elems<P1, T>();  // holds U, then ur / wr
+    T* bS = bR0 + CF::BUF;
     T* bT = bS + CF::BUF;
     load_op<P1, T, NT>(opD, D);
     load_op<P1, T, NT, true>(opT, D);
@@ -525,7 +646,7 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
         const int nlines = ne * P1 * P1;
         const int64_t gbase = e0 * G::NPTS;
         __syncthreads();
-        load_group_async<P1, P1, T, NT>(bR, Uin + gbase, ne);
+        T* bR = load_group_async<P1, P1, T, NT>(bR0, Uin + gbase, ne);
         cp_async_commit();
         cp_async_wait_all();
         __syncthreads();

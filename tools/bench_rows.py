@@ -67,7 +67,21 @@ def spectral(p, N, dims):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--sections", default="cfg1,cfg5,cfg2,ccsdt", help="comma list of cfg1,cfg5,cfg2,ccsdt")
+    ap.add_argument("--tiles", default="16,24")
     args = ap.parse_args()
+    sec = set(args.sections.split(","))
+    if "cfg1" in sec:
+        cfg1()
+    if "cfg5" in sec:
+        cfg5(args)
+    if "cfg2" in sec:
+        cfg2()
+    if "ccsdt" in sec:
+        ccsdt(args)
+
+
+def cfg1():
 
     # ---- config 1: 3-D p=4, N=64 (latency-bound by construction): per call and graph-amortised
     P1, U, A, B, C = spectral(4, 64, 3)
@@ -87,6 +101,9 @@ def main():
     emit("sumfact3d", "cfg1 p=4 N=64", ms, mean, 6 * P1 ** 4 * 64, 16 * P1 ** 3 * 64, 64, "elements_per_s",
          {"graph_us_per_call": round(gms * 1e3 / 1000, 3), "note": "HBM time 16 ns: launch/latency-bound"})
 
+
+
+def cfg5(args):
     # ---- config 5: spectral sweep p = 4..12, N = 2^16 .. 2^22, 3-D and 2-D
     ps = [4, 8, 12] if args.quick else [4, 5, 6, 7, 8, 9, 10, 11, 12]
     Ns = [2 ** 20] if args.quick else [2 ** 16, 2 ** 18, 2 ** 20, 2 ** 22]
@@ -109,6 +126,9 @@ def main():
             del U, V
             torch.cuda.empty_cache()
 
+
+
+def cfg2():
     # ---- config 2: local_grad3 p=12 N=262144, and the NEXT rows at the same size
     p, N = 12, 262144
     P1, U, A, B, C = spectral(p, N, 3)
@@ -131,8 +151,11 @@ def main():
     del U, W, Gm, Ug, Wg
     torch.cuda.empty_cache()
 
+
+
+def ccsdt(args):
     # ---- configs 3 / 4: CCSD(T) per-variant and fused, tiles 16 and 24 (s1: NEXT f3)
-    for t in ([16] if args.quick else [16, 24]):
+    for t in ([16] if args.quick else [int(x) for x in args.tiles.split(",")]):
         ext = (t,) * 7
         t3 = bc.fill(torch.empty(t ** 6, dtype=torch.float64, device=DEV), 10)
         ops = {f: ([bc.fill(torch.empty(t ** 4, dtype=torch.float64, device=DEV), 20 + v) for v in range(9)],
