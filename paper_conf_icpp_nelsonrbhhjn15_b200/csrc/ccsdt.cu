@@ -1636,19 +1636,23 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
 // loads in flight at once.  Per element and entry: 2 shared loads and one FMA; the hole
 // names of an element are linear forms of its storage coordinates, one per class.
 // ==================================================================================
-constexpr int S1S_NT = 256, S1S_U = 8;  // threads, t3 values in flight per thread
+constexpr int S1S_NT = 256, S1S_U = 4;  // threads, runs in flight per thread
 
+// RUN consecutive storage-position-0 values per thread (16-byte accesses when RUN = 4).
+// Shared layout per class c (CS doubles): V_c[pair][m] (pair = h2 (H3+1) + h3) then
+// T_c[h1][m], m = the entry's rank inside its class, so one address per class serves its
+// (up to 3) entries through immediate offsets.
+template <int RUN>
 __global__ void __launch_bounds__(S1S_NT) ccsdt_s1_stream_kernel(const __grid_constant__ CcsdtParams P,
                                                                  int nplanes) {
     extern __shared__ __align__(16) double s1sm[];
     const int H1 = P.ext[N_H1], H2 = P.ext[N_H2], H3 = P.ext[N_H3];
     const int P4 = P.ext[N_P4], P6 = P.ext[N_P6];
-    const int VS = H2 * (H3 + 1), ES = VS + H1;   // per entry: Vs [h2][h3] (row stride H3+1), Ts [h1]
-    const int BUFD = P.nentry * ES;               // one plane's factors (2 buffers)
+    const int VS = H2 * (H3 + 1), CS = 3 * (VS + H1);
+    const int BUFD = P.ncls * CS;
     const int Q0 = P.qe[0], Q1 = P.qe[1], Q2 = P.qe[2];
-    const int nh = Q0 * Q1 * Q2;
+    const int nh = Q0 * Q1 * Q2, R0 = Q0 / RUN, nruns = nh / RUN;
     const int tid = threadIdx.x;
-    // entries are grouped by class (run_ccsdt): slot (c, m) = entry cb[c] + m, m < cnt[c]
     int n0 = 0, n1 = 0, n2 = 0;
     for (int e = 0; e < P.nentry; ++e) {
         const int c = P.ecls[e];
@@ -1657,104 +1661,162 @@ __global__ void __launch_bounds__(S1S_NT) ccsdt_s1_stream_kernel(const __grid_co
         n2 += c == 2;
     }
     const int cb[3] = {0, n0, n0 + n1}, cnt[3] = {n0, n1, n2};
-    uint32_t sm_[3][3];
     int av[3][3], at[3][3];
 #pragma unroll
-    for (int c = 0; c < 3; ++c) {
-#pragma unroll
-        for (int m = 0; m < 3; ++m) sm_[c][m] = (m < cnt[c]) ? P.smask[cb[c] + m] : 0u;
+    for (int c = 0; c < 3; ++c)
 #pragma unroll
         for (int q = 0; q < 3; ++q) {
             const bool ok = c < P.ncls;
             at[c][q] = (ok && P.hpos[c][0] == q) ? 1 : 0;                                            // h1
             av[c][q] = (ok && P.hpos[c][1] == q) ? H3 + 1 : ((ok && P.hpos[c][2] == q) ? 1 : 0);  // h2, h3
         }
-    }
-    // stage plane j's factors into buffer b (cp.async; signs are applied at use)
-    auto stage = [&](int plane, int b) {
+    auto pvals = [&](int plane, int e, int& p4, int& p5, int& p6) {
         const int qv0 = plane % P.qe[3], qv1 = (plane / P.qe[3]) % P.qe[4], qv2 = plane / (P.qe[3] * P.qe[4]);
         auto pick = [&](int pos) { return pos == 3 ? qv0 : (pos == 4 ? qv1 : qv2); };
+        p4 = pick(P.ppos[e][0]);
+        p5 = pick(P.ppos[e][1]);
+        p6 = pick(P.ppos[e][2]);
+    };
+    // V factors of a plane: cp.async into buffer b
+    auto stage_v = [&](int plane, int b) {
         double* buf = s1sm + b * BUFD;
         for (int e = 0; e < P.nentry; ++e) {
-            const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
+            int p4, p5, p6;
+            pvals(plane, e, p4, p5, p6);
+            const int c = P.ecls[e], m = e - (c == 0 ? 0 : (c == 1 ? n0 : n0 + n1));
             const double* v2 = P.opB[e] + (int64_t)H3 * H2 * (p6 + (int64_t)P6 * p5);
+            double* dst = buf + c * CS + m;
             for (int i = tid; i < H2 * H3; i += S1S_NT) {
                 const int h2 = i / H3, h3 = i - h2 * H3;
-                cp_async_8(buf + e * ES + h2 * (H3 + 1) + h3, v2 + i);
+                cp_async_8(dst + 3 * (h2 * (H3 + 1) + h3), v2 + i);
             }
-            const double* t1 = P.opA[e] + p4;
-            for (int h1 = tid; h1 < H1; h1 += S1S_NT) cp_async_8(buf + e * ES + VS + h1, t1 + (int64_t)P4 * h1);
         }
     };
-    // this thread's storage coordinates at i = tid and the step for i += S1S_NT
-    const int iq0 = tid % Q0, iq1 = (tid / Q0) % Q1, iq2 = tid / (Q0 * Q1);
-    const int d0 = S1S_NT % Q0, d1 = (S1S_NT / Q0) % Q1, d2 = S1S_NT / (Q0 * Q1);
+    // T factors (sign folded): thread t < nentry*H1 owns one value; loaded one plane ahead
+    const int te = tid / (H1 > 0 ? H1 : 1), th1 = tid - te * H1;
+    const bool towner = te < P.nentry;
+    const int tc = towner ? P.ecls[te] : 0;
+    const int tdst = tc * CS + 3 * VS + 3 * th1 + (te - (tc == 0 ? 0 : (tc == 1 ? n0 : n0 + n1)));
+    const double tsg = towner ? P.sign[te] : 0.0;
+    auto load_t = [&](int plane) {
+        if (!towner) return 0.0;
+        int p4, p5, p6;
+        pvals(plane, te, p4, p5, p6);
+        return __ldg(P.opA[te] + p4 + (int64_t)P4 * th1);
+    };
+    const bool t_fast = P.nentry * H1 <= S1S_NT;
+    auto stage_t_slow = [&](int plane, int b) {  // more T values than threads
+        double* buf = s1sm + b * BUFD;
+        for (int i = tid; i < P.nentry * H1; i += S1S_NT) {
+            const int e = i / H1, h1 = i - e * H1;
+            int p4, p5, p6;
+            pvals(plane, e, p4, p5, p6);
+            const int c = P.ecls[e], m = e - (c == 0 ? 0 : (c == 1 ? n0 : n0 + n1));
+            buf[c * CS + 3 * VS + 3 * h1 + m] = P.sign[e] * __ldg(P.opA[e] + p4 + (int64_t)P4 * h1);
+        }
+    };
+    // this thread's run coordinates at run index tid, and the step for += S1S_NT runs
+    const int iq0 = tid % R0, iq1 = (tid / R0) % Q1, iq2 = tid / (R0 * Q1);
+    const int d0 = S1S_NT % R0, d1 = (S1S_NT / R0) % Q1, d2 = S1S_NT / (R0 * Q1);
+
     int it = 0;
-    if ((int)blockIdx.x < nplanes) stage(blockIdx.x, 0);
+    if ((int)blockIdx.x < nplanes) {
+        stage_v(blockIdx.x, 0);
+        if (t_fast) {
+            if (towner) s1sm[tdst] = tsg * load_t(blockIdx.x);
+        } else {
+            stage_t_slow(blockIdx.x, 0);
+        }
+    }
     cp_async_commit();
     for (int plane = blockIdx.x; plane < nplanes; plane += gridDim.x, ++it) {
         cp_async_wait_all();
-        __syncthreads();  // this plane's factors landed; the other buffer is free
-        if (plane + (int)gridDim.x < nplanes) stage(plane + gridDim.x, (it + 1) & 1);
+        __syncthreads();  // this plane's factors are in place; the other buffer is free
+        const int nxt = plane + gridDim.x;
+        double tnext = 0.0;
+        if (nxt < nplanes) {
+            stage_v(nxt, (it + 1) & 1);
+            if (t_fast) tnext = load_t(nxt);
+            else stage_t_slow(nxt, (it + 1) & 1);
+        }
         cp_async_commit();
         const double* buf = s1sm + (it & 1) * BUFD;
         double* t3p = P.t3 + (int64_t)nh * plane;
         int q0 = iq0, q1 = iq1, q2 = iq2;
-        for (int i0 = 0; i0 < nh; i0 += S1S_NT * S1S_U) {
-            double x[S1S_U];
+        for (int r0 = 0; r0 < nruns; r0 += S1S_NT * S1S_U) {
+            double x[S1S_U][RUN];
 #pragma unroll
             for (int u = 0; u < S1S_U; ++u) {
-                const int i = i0 + u * S1S_NT + tid;
-                x[u] = (i < nh) ? __ldcs(t3p + i) : 0.0;
+                const int r = r0 + u * S1S_NT + tid;
+                if (r < nruns) {
+                    if constexpr (RUN == 4) {
+                        const double2 a = __ldcs(reinterpret_cast<const double2*>(t3p) + 2 * r);
+                        const double2 b = __ldcs(reinterpret_cast<const double2*>(t3p) + 2 * r + 1);
+                        x[u][0] = a.x; x[u][1] = a.y; x[u][2] = b.x; x[u][3] = b.y;
+                    } else {
+                        x[u][0] = __ldcs(t3p + r);
+                    }
+                }
             }
 #pragma unroll
             for (int u = 0; u < S1S_U; ++u) {
-                const int i = i0 + u * S1S_NT + tid;
-                if (i < nh) {
-                    double acc = x[u];
+                const int r = r0 + u * S1S_NT + tid;
+                if (r < nruns) {
+                    const int qq0 = q0 * RUN;
 #pragma unroll
                     for (int c = 0; c < 3; ++c) {
-                        const int vo = q0 * av[c][0] + q1 * av[c][1] + q2 * av[c][2];
-                        const int to = VS + q0 * at[c][0] + q1 * at[c][1] + q2 * at[c][2];
+                        if (c < P.ncls) {
+                            const double* Vc = buf + c * CS + 3 * (qq0 * av[c][0] + q1 * av[c][1] + q2 * av[c][2]);
+                            const double* Tc = buf + c * CS + 3 * (VS + qq0 * at[c][0] + q1 * at[c][1] + q2 * at[c][2]);
+                            const int dv = 3 * av[c][0], dt = 3 * at[c][0];
 #pragma unroll
-                        for (int m = 0; m < 3; ++m)
-                            if (m < cnt[c]) {
-                                const double* eb = buf + (cb[c] + m) * ES;
-                                acc = fma(flip_sign(eb[to], sm_[c][m]), eb[vo], acc);
-                            }
+                            for (int k = 0; k < RUN; ++k)
+#pragma unroll
+                                for (int m = 0; m < 3; ++m)
+                                    if (m < cnt[c]) x[u][k] = fma(Tc[k * dt + m], Vc[k * dv + m], x[u][k]);
+                        }
                     }
-                    __stcs(t3p + i, acc);
+                    if constexpr (RUN == 4) {
+                        __stcs(reinterpret_cast<double2*>(t3p) + 2 * r, make_double2(x[u][0], x[u][1]));
+                        __stcs(reinterpret_cast<double2*>(t3p) + 2 * r + 1, make_double2(x[u][2], x[u][3]));
+                    } else {
+                        __stcs(t3p + r, x[u][0]);
+                    }
                 }
-                // advance (q0, q1, q2) by S1S_NT elements
                 q0 += d0;
-                const int c0 = q0 >= Q0;
-                q0 -= c0 ? Q0 : 0;
+                const int c0 = q0 >= R0;
+                q0 -= c0 ? R0 : 0;
                 q1 += d1 + c0;
                 const int c1 = q1 >= Q1;
                 q1 -= c1 ? Q1 : 0;
                 q2 += d2 + c1;
             }
         }
+        if (t_fast && towner && nxt < nplanes) s1sm[((it + 1) & 1) * BUFD + tdst] = tsg * tnext;
     }
 }
 
 static int launch_ccsdt_s1_stream(const CcsdtParams& P, cudaStream_t s) {
-    const size_t smem = 2 * ((size_t)P.nentry * (P.ext[N_H2] * (P.ext[N_H3] + 1) + P.ext[N_H1])) * 8;
+    const size_t smem = 2 * ((size_t)P.ncls * 3 * (P.ext[N_H2] * (P.ext[N_H3] + 1) + P.ext[N_H1])) * 8;
     if (smem > 200 * 1024) return 1;
     const int nplanes = P.qe[3] * P.qe[4] * P.qe[5];
     if (nplanes == 0 || P.qe[0] * P.qe[1] * P.qe[2] == 0) return BC_OK;
-    static size_t last_smem = 0;
-    static int occ = 0;
-    if (smem != last_smem) {
-        cudaFuncSetAttribute(ccsdt_s1_stream_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_s1_stream_kernel, S1S_NT, smem);
-        if (occ < 1) occ = 1;
-        last_smem = smem;
-    }
-    const int64_t cap = (int64_t)num_sms() * occ;
-    const int grid = (int)(nplanes < cap ? nplanes : cap);
-    ccsdt_s1_stream_kernel<<<grid, S1S_NT, smem, s>>>(P, nplanes);
-    return launch_status();
+    const bool run4 = P.qe[0] % 4 == 0;
+    auto go = [&](auto kern, size_t* last_smem, int* occ) {
+        if (smem != *last_smem) {
+            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, kern, S1S_NT, smem);
+            if (*occ < 1) *occ = 1;
+            *last_smem = smem;
+        }
+        const int64_t cap = (int64_t)num_sms() * *occ;
+        const int grid = (int)(nplanes < cap ? nplanes : cap);
+        kern<<<grid, S1S_NT, smem, s>>>(P, nplanes);
+        return launch_status();
+    };
+    static size_t ls4 = 0, ls1 = 0;
+    static int occ4 = 0, occ1 = 0;
+    return run4 ? go(ccsdt_s1_stream_kernel<4>, &ls4, &occ4) : go(ccsdt_s1_stream_kernel<1>, &ls1, &occ1);
 }
 
 // ==================================================================================
@@ -1853,17 +1915,27 @@ __global__ void __launch_bounds__(SV_NT, 2) ccsdt_sv16_kernel(const __grid_const
         names(j, a, o1, o2);
         if (a != curA) {
             __syncthreads();  // every thread is done with the previous A
-            if (FAM == FAM_D1) {  // As[k][h2][h3] = s v2[h3,h2,p6,k]
+            if (FAM == FAM_D1) {  // As[k][h2][h3] = v2[h3,h2,p6,k]: 16-byte copies
                 const double* src = opB + 256LL * a;
-                for (int i = tid; i < 256 * K; i += SV_NT) {
-                    const int k = i >> 8, r = i & 255;
-                    As[k * SV_PS + (r >> 4) * SV_RS + (r & 15)] = sg * __ldg(src + (int64_t)256 * P6 * k + r);
+                for (int i = tid; i < 128 * K; i += SV_NT) {
+                    const int k = i >> 7, r = 2 * (i & 127);
+                    cp_async_16(As + k * SV_PS + (r >> 4) * SV_RS + (r & 15), src + (int64_t)256 * P6 * k + r);
                 }
-            } else {  // As[k][h1][h2] = s t2[k,p4,h1,h2]
+            } else {  // As[k][h1][h2] = t2[k,p4,h1,h2]
                 const double* src = opA + (int64_t)K * a;
                 for (int i = tid; i < 256 * K; i += SV_NT) {
                     const int r = i / K, k = i - r * K;  // r = h1 + 16 h2
-                    As[k * SV_PS + (r & 15) * SV_RS + (r >> 4)] = sg * __ldg(src + (int64_t)K * P4 * r + k);
+                    cp_async_8(As + k * SV_PS + (r & 15) * SV_RS + (r >> 4), src + (int64_t)K * P4 * r + k);
+                }
+            }
+            cp_async_commit();
+            if (sg < 0.0) {  // fold the variant's sign into A once (exact)
+                cp_async_wait_all();
+                __syncthreads();
+                for (int i = tid; i < 256 * K; i += SV_NT) {
+                    const int k = i >> 8, r = i & 255;
+                    double& v = As[k * SV_PS + (r >> 4) * SV_RS + (r & 15)];
+                    v = -v;
                 }
             }
             curA = a;
@@ -1906,8 +1978,224 @@ __global__ void __launch_bounds__(SV_NT, 2) ccsdt_sv16_kernel(const __grid_const
     }
 }
 
+// ---- sv16 with the Tensor Memory Accelerator streaming the t3 planes (BC_SV16_BULK=1;
+// measured on par with / slightly below the register-streamed kernel above).
+// One persistent CTA per SM.  Thread 0 keeps SVB_PF planes of bulk copies
+// (cp.async.bulk, 32 KB each, mbarrier completion) in flight into a ring of SVB_NS plane
+// buffers; the threads read their 4 x 4 tile from the buffer, accumulate, write it back,
+// and thread 0 bulk-stores the plane (bulk_group; a buffer is reloaded only after the
+// store that last read it has finished reading).  Memory parallelism no longer depends on
+// registers: ~64 KB of loads plus the stores in flight per SM.  Tile reads/writes are
+// conflict-free: odd-`bo` lanes touch their row's second 16-byte half first.
+constexpr int SVB_NS = 4, SVB_PF = 2;
+
+__device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, int bytes, uint32_t bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n"
+                 ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void bulk_store(void* dst, uint32_t src, int bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;\n" ::"l"(dst), "r"(src), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;\n" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+    asm volatile("cp.async.bulk.wait_group.read %0;\n" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;\n" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory"); }
+
+template <int FAM>
+__global__ void __launch_bounds__(SV_NT, 1) ccsdt_sv16b_kernel(const __grid_constant__ CcsdtParams P, int nplanes) {
+    extern __shared__ __align__(16) double svsm[];
+    const int K = P.ext[N_K];
+    double* ring = svsm;                          // SVB_NS planes of 4096
+    double* As = ring + SVB_NS * 4096;            // [k][f][x]
+    double* Bs = As + K * SV_PS;                  // SVB_NS buffers of [k][y]
+    uint64_t* bars = reinterpret_cast<uint64_t*>(Bs + SVB_NS * 16 * K);
+    const uint32_t bar0 = smem_u32(bars), ring0 = smem_u32(ring);
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int* hp = P.hpos[0];
+    const int posX = (FAM == FAM_D1) ? hp[2] : hp[1];
+    const int posY = (FAM == FAM_D1) ? hp[0] : hp[2];
+    const int posF = (FAM == FAM_D1) ? hp[1] : hp[0];
+    const bool xfast = posX == 0;
+    const int bq = lane & 3, bo = (lane >> 2) & 3;
+    const int bx = xfast ? bq : bo, by = xfast ? bo : bq;
+    const int f = 2 * warp + (lane >> 4);
+    const int sX = 1 << (4 * posX), sY = 1 << (4 * posY), sF = 1 << (4 * posF);
+    const int rstride = xfast ? sY : sX;
+    const int tbase = 4 * bx * sX + 4 * by * sY + f * sF;
+    const bool sw = bo & 1;                      // odd bo: second 16-byte half first (no bank conflicts)
+    const int h0 = sw ? 2 : 0, h1o = 2 - h0;
+    const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6];
+    const int PO1 = (FAM == FAM_D1) ? P5 : P6, PO2 = (FAM == FAM_D1) ? P4 : P5;
+    auto qstride = [&](int pos) {
+        return pos == 3 ? 4096LL : (pos == 4 ? 4096LL * P.qe[3] : 4096LL * P.qe[3] * P.qe[4]);
+    };
+    const int64_t sp4 = qstride(P.ppos[0][0]), sp5 = qstride(P.ppos[0][1]), sp6 = qstride(P.ppos[0][2]);
+    const double sg = P.sign[0];
+    const double* __restrict__ opA = P.opA[0];
+    const double* __restrict__ opB = P.opB[0];
+    const int lo = (int)((int64_t)nplanes * blockIdx.x / gridDim.x);
+    const int hi = (int)((int64_t)nplanes * (blockIdx.x + 1) / gridDim.x);
+    const int n = hi - lo;
+    auto names = [&](int j, int& a, int& o1, int& o2) {
+        a = j / (PO1 * PO2);
+        const int r = j - a * (PO1 * PO2);
+        o1 = r / PO2;
+        o2 = r - o1 * PO2;
+    };
+    auto plane_ptr = [&](int j) {
+        int a, o1, o2;
+        names(j, a, o1, o2);
+        const int p4 = (FAM == FAM_D1) ? o2 : a, p5 = (FAM == FAM_D1) ? o1 : o2, p6 = (FAM == FAM_D1) ? a : o1;
+        return P.t3 + p4 * sp4 + p5 * sp5 + p6 * sp6;
+    };
+    auto issue_B = [&](int j, double* dst) {
+        int a, o1, o2;
+        names(j, a, o1, o2);
+        const double* src = (FAM == FAM_D1) ? opA + (int64_t)K * (o2 + (int64_t)P4 * o1)
+                                            : opB + (int64_t)K * 16 * (o1 + (int64_t)P6 * o2);
+        const int stride_y = (FAM == FAM_D1) ? K * P4 * P5 : K;
+        for (int i = tid; i < 16 * K; i += SV_NT) {
+            const int y = i / K, k = i - y * K;
+            cp_async_8(dst + k * 16 + y, src + (int64_t)stride_y * y + k);
+        }
+    };
+    if (n <= 0) return;
+    if (tid == 0) {
+        for (int i = 0; i < SVB_NS; ++i) mbar_init(bar0 + 8 * i, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    __syncthreads();
+    // prologue: t3 planes lo .. lo+PF-1 (bulk) and their B slices (one cp.async group each)
+    for (int i = 0; i < SVB_PF; ++i) {
+        if (i < n) {
+            if (tid == 0) {
+                mbar_expect_tx(bar0 + 8 * i, 32768);
+                bulk_load(ring0 + i * 32768, plane_ptr(lo + i), 32768, bar0 + 8 * i);
+            }
+            issue_B(lo + i, Bs + i * 16 * K);
+        }
+        cp_async_commit();
+    }
+    int curA = -1;
+    for (int idx = 0; idx < n; ++idx) {
+        const int j = lo + idx, s = idx % SVB_NS;
+        int a, o1, o2;
+        names(j, a, o1, o2);
+        if (a != curA) {  // stage A (sign folded) — once or twice per CTA
+            __syncthreads();
+            if (FAM == FAM_D1) {  // As[k][h2][h3] = v2[h3,h2,p6,k]: 16-byte copies
+                const double* src = opB + 256LL * a;
+                for (int i = tid; i < 128 * K; i += SV_NT) {
+                    const int k = i >> 7, r = 2 * (i & 127);
+                    cp_async_16(As + k * SV_PS + (r >> 4) * SV_RS + (r & 15), src + (int64_t)256 * P6 * k + r);
+                }
+            } else {  // As[k][h1][h2] = t2[k,p4,h1,h2]
+                const double* src = opA + (int64_t)K * a;
+                for (int i = tid; i < 256 * K; i += SV_NT) {
+                    const int r = i / K, k = i - r * K;
+                    cp_async_8(As + k * SV_PS + (r & 15) * SV_RS + (r >> 4), src + (int64_t)K * P4 * r + k);
+                }
+            }
+            cp_async_commit();
+            cp_async_wait_n<0>();
+            if (sg < 0.0) {  // fold the sign into A (exact)
+                __syncthreads();
+                for (int i = tid; i < 256 * K; i += SV_NT) {
+                    double& v = As[(i >> 8) * SV_PS + ((i & 255) >> 4) * SV_RS + (i & 15)];
+                    v = -v;
+                }
+            }
+            curA = a;
+        }
+        cp_async_wait_n<SVB_PF - 1>();                 // this thread's B(j) copies landed
+        mbar_wait(bar0 + 8 * s, (idx / SVB_NS) & 1);   // t3 plane j landed
+        __syncthreads();                               // all B(j), A visible
+        // refill: plane j+PF into the buffer plane j+PF-NS used (its store has read it)
+        if (idx + SVB_PF < n) {
+            const int s2 = (idx + SVB_PF) % SVB_NS;
+            if (tid == 0) {
+                bulk_wait_read<SVB_NS - SVB_PF - 1>();
+                fence_proxy_async();
+                mbar_expect_tx(bar0 + 8 * s2, 32768);
+                bulk_load(ring0 + s2 * 32768, plane_ptr(j + SVB_PF), 32768, bar0 + 8 * s2);
+            }
+            issue_B(j + SVB_PF, Bs + s2 * 16 * K);
+        }
+        cp_async_commit();
+        double* buf = ring + s * 4096 + tbase;
+        double acc[4][4];
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            const double2 u = *reinterpret_cast<const double2*>(buf + r * rstride + h0);
+            const double2 w = *reinterpret_cast<const double2*>(buf + r * rstride + h1o);
+            acc[r][0] = sw ? w.x : u.x;
+            acc[r][1] = sw ? w.y : u.y;
+            acc[r][2] = sw ? u.x : w.x;
+            acc[r][3] = sw ? u.y : w.y;
+        }
+        const double* Ap = As + f * SV_RS + 4 * bx;
+        const double* Bp = Bs + s * 16 * K + 4 * by;
+#pragma unroll 4
+        for (int k = 0; k < K; ++k) {
+            const double2 a01 = *reinterpret_cast<const double2*>(Ap + k * SV_PS);
+            const double2 a23 = *reinterpret_cast<const double2*>(Ap + k * SV_PS + 2);
+            const double2 b01 = *reinterpret_cast<const double2*>(Bp + k * 16);
+            const double2 b23 = *reinterpret_cast<const double2*>(Bp + k * 16 + 2);
+            const double av[4] = {a01.x, a01.y, a23.x, a23.y}, bv[4] = {b01.x, b01.y, b23.x, b23.y};
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+#pragma unroll
+                for (int jj = 0; jj < 4; ++jj) {
+                    double& t = xfast ? acc[jj][i] : acc[i][jj];
+                    t = fma(av[i], bv[jj], t);
+                }
+        }
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            *reinterpret_cast<double2*>(buf + r * rstride + h0) =
+                sw ? make_double2(acc[r][2], acc[r][3]) : make_double2(acc[r][0], acc[r][1]);
+            *reinterpret_cast<double2*>(buf + r * rstride + h1o) =
+                sw ? make_double2(acc[r][0], acc[r][1]) : make_double2(acc[r][2], acc[r][3]);
+        }
+        fence_proxy_async();  // generic-proxy writes -> visible to the bulk store
+        __syncthreads();
+        if (tid == 0) {
+            bulk_store(plane_ptr(j), ring0 + s * 32768, 32768);
+            bulk_commit();
+        }
+    }
+    if (tid == 0) bulk_wait_all();
+}
+
+template <int FAM>
+static int launch_ccsdt_sv16b(const CcsdtParams& P, cudaStream_t s) {
+    const int K = P.ext[N_K];
+    const size_t smem = ((size_t)SVB_NS * 4096 + (size_t)K * SV_PS + (size_t)SVB_NS * 16 * K) * 8 + SVB_NS * 8;
+    if (smem > 227 * 1024) return 1;
+    const int nplanes = P.qe[3] * P.qe[4] * P.qe[5];
+    if (nplanes == 0) return BC_OK;
+    static bool init = false;
+    if (!init) {
+        cudaFuncSetAttribute(ccsdt_sv16b_kernel<FAM>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+        init = true;
+    }
+    const int grid = nplanes < num_sms() ? nplanes : num_sms();
+    ccsdt_sv16b_kernel<FAM><<<grid, SV_NT, smem, s>>>(P, nplanes);
+    return launch_status();
+}
+
 template <int FAM>
 static int launch_ccsdt_sv16(const CcsdtParams& P, cudaStream_t s) {
+    // register-streamed kernel by default (tile 16, back-to-back calls: 0.63-0.67 of HBM vs
+    // 0.62-0.63 for the bulk-streamed one, 0.56-0.57 for the TMA cube kernel)
+    if (getenv("BC_SV16_BULK") != nullptr) {
+        const int st = launch_ccsdt_sv16b<FAM>(P, s);
+        if (st != 1) return st;
+    }
     const int K = P.ext[N_K];
     const size_t smem = ((size_t)K * SV_PS + 2 * 16 * (size_t)K) * 8;
     const int nplanes = P.qe[3] * P.qe[4] * P.qe[5];
