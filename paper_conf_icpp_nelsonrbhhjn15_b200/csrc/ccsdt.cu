@@ -1637,13 +1637,16 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
 // names of an element are linear forms of its storage coordinates, one per class.
 // ==================================================================================
 constexpr int S1S_NT = 256, S1S_U = 4;  // threads, runs in flight per thread
+#ifndef BC_S1_MINB
+#define BC_S1_MINB 1  // measured: 3 or 4 CTAs/SM (79 / 64 registers) are slower than 2 (128 registers)
+#endif
 
 // RUN consecutive storage-position-0 values per thread (16-byte accesses when RUN = 4).
 // Shared layout per class c (CS doubles): V_c[pair][m] (pair = h2 (H3+1) + h3) then
 // T_c[h1][m], m = the entry's rank inside its class, so one address per class serves its
 // (up to 3) entries through immediate offsets.
 template <int RUN>
-__global__ void __launch_bounds__(S1S_NT) ccsdt_s1_stream_kernel(const __grid_constant__ CcsdtParams P,
+__global__ void __launch_bounds__(S1S_NT, BC_S1_MINB) ccsdt_s1_stream_kernel(const __grid_constant__ CcsdtParams P,
                                                                  int nplanes) {
     extern __shared__ __align__(16) double s1sm[];
     const int H1 = P.ext[N_H1], H2 = P.ext[N_H2], H3 = P.ext[N_H3];
@@ -1842,59 +1845,74 @@ __device__ __forceinline__ void st_cs2(double* p, double a, double b) {
     __stcs(reinterpret_cast<double2*>(p), make_double2(a, b));
 }
 
-template <int FAM>
-__global__ void __launch_bounds__(SV_NT, 2) ccsdt_sv16_kernel(const __grid_constant__ CcsdtParams P, int nplanes) {
+// Geometry per hole extent H: a unit is (particle plane, range of NF values of f); thread
+// tiles are 4 x 4 over (x, y), so a unit has (H/4)^2 NF tiles = NT threads.
+template <int H>
+struct SvGeo {
+    static constexpr int NB = H / 4;               // tile blocks per hole axis
+    static constexpr int NF = H == 16 ? 16 : 4;    // f values per unit
+    static constexpr int NT = NB * NB * NF;        // 256 | 144
+    static constexpr int MINB = H == 16 ? 2 : 3;   // CTAs per SM (128 registers)
+    static constexpr int NFR = H / NF;             // units per plane: 1 | 6
+    static constexpr int RS = H + 2;               // A row stride (doubles, even)
+    static constexpr int PS = NF * RS + 2;         // A k-plane stride
+};
+
+template <int FAM, int H>
+__global__ void __launch_bounds__(SvGeo<H>::NT, SvGeo<H>::MINB) ccsdt_svs_kernel(const __grid_constant__ CcsdtParams P, int nunits) {
+    using G = SvGeo<H>;
+    constexpr int NB = G::NB, NF = G::NF, NT = G::NT, RS = G::RS, PS = G::PS, NFR = G::NFR;
     extern __shared__ __align__(16) double svsm[];
     const int K = P.ext[N_K];
-    double* As = svsm;                 // [k][f][x] (row stride SV_RS, k-plane stride SV_PS)
-    double* Bs = As + K * SV_PS;       // 2 buffers of [k][y]
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    double* As = svsm;                 // [k][fl][x]
+    double* Bs = As + K * PS;          // 2 buffers of [k][y]
+    const int tid = threadIdx.x;
+    const int bq = tid % NB, bo = (tid / NB) % NB, fl = tid / (NB * NB);
     const int* hp = P.hpos[0];         // storage positions of h1, h2, h3
     const int posX = (FAM == FAM_D1) ? hp[2] : hp[1];
     const int posY = (FAM == FAM_D1) ? hp[0] : hp[2];
     const int posF = (FAM == FAM_D1) ? hp[1] : hp[0];
     const bool xfast = posX == 0;      // else posY == 0
-    const int bq = lane & 3, bo = (lane >> 2) & 3;
     const int bx = xfast ? bq : bo, by = xfast ? bo : bq;
-    const int f = 2 * warp + (lane >> 4);
-    const int sX = 1 << (4 * posX), sY = 1 << (4 * posY), sF = 1 << (4 * posF);
-    // the tile's 4 rows of 4 contiguous values: row r -> offset, element c contiguous
+    auto hstride = [](int pos) { return pos == 0 ? 1 : (pos == 1 ? H : H * H); };
+    const int sX = hstride(posX), sY = hstride(posY), sF = hstride(posF);
     const int rstride = xfast ? sY : sX;
-    const int tbase = 4 * bx * sX + 4 * by * sY + f * sF;
-    // particle names: A name a (d1 p6, d2 p4) slowest, then o1, o2
+    const int tbase = 4 * bx * sX + 4 * by * sY + fl * sF;
     const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6];
     const int PO1 = (FAM == FAM_D1) ? P5 : P6, PO2 = (FAM == FAM_D1) ? P4 : P5;
+    constexpr int64_t HV = (int64_t)H * H * H;
     auto qstride = [&](int pos) {
-        return pos == 3 ? 4096LL : (pos == 4 ? 4096LL * P.qe[3] : 4096LL * P.qe[3] * P.qe[4]);
+        return pos == 3 ? HV : (pos == 4 ? HV * P.qe[3] : HV * P.qe[3] * P.qe[4]);
     };
     const int64_t sp4 = qstride(P.ppos[0][0]), sp5 = qstride(P.ppos[0][1]), sp6 = qstride(P.ppos[0][2]);
     const double sg = P.sign[0];
     const double* __restrict__ opA = P.opA[0];  // t2
     const double* __restrict__ opB = P.opB[0];  // v2
-
-    const int lo = (int)((int64_t)nplanes * blockIdx.x / gridDim.x);
-    const int hi = (int)((int64_t)nplanes * (blockIdx.x + 1) / gridDim.x);
-    auto names = [&](int j, int& a, int& o1, int& o2) {
-        a = j / (PO1 * PO2);
-        const int r = j - a * (PO1 * PO2);
+    const int lo = (int)((int64_t)nunits * blockIdx.x / gridDim.x);
+    const int hi = (int)((int64_t)nunits * (blockIdx.x + 1) / gridDim.x);
+    // unit u -> (a, fr, o1, o2), a = the A name (d1 p6, d2 p4) slowest
+    auto decode = [&](int u, int& akey, int& o1, int& o2) {
+        akey = u / (PO1 * PO2);  // a * NFR + fr
+        const int r = u - akey * (PO1 * PO2);
         o1 = r / PO2;
         o2 = r - o1 * PO2;
     };
-    auto plane_ptr = [&](int j) {
-        int a, o1, o2;
-        names(j, a, o1, o2);
+    auto unit_ptr = [&](int u) {
+        int akey, o1, o2;
+        decode(u, akey, o1, o2);
+        const int a = akey / NFR, fr = akey - a * NFR;
         const int p4 = (FAM == FAM_D1) ? o2 : a, p5 = (FAM == FAM_D1) ? o1 : o2, p6 = (FAM == FAM_D1) ? a : o1;
-        return P.t3 + p4 * sp4 + p5 * sp5 + p6 * sp6 + tbase;
+        return P.t3 + p4 * sp4 + p5 * sp5 + p6 * sp6 + fr * NF * sF + tbase;
     };
-    auto issue_B = [&](int j, double* dst) {  // B[k][y], 16 K values
-        int a, o1, o2;
-        names(j, a, o1, o2);
+    auto issue_B = [&](int u, double* dst) {  // B[k][y]
+        int akey, o1, o2;
+        decode(u, akey, o1, o2);
         const double* src = (FAM == FAM_D1) ? opA + (int64_t)K * (o2 + (int64_t)P4 * o1)       // t2[k,p4,p5,h1]
-                                            : opB + (int64_t)K * 16 * (o1 + (int64_t)P6 * o2);  // v2[k,h3,p6,p5]
+                                            : opB + (int64_t)K * H * (o1 + (int64_t)P6 * o2);  // v2[k,h3,p6,p5]
         const int stride_y = (FAM == FAM_D1) ? K * P4 * P5 : K;
-        for (int i = tid; i < 16 * K; i += SV_NT) {
+        for (int i = tid; i < H * K; i += NT) {
             const int y = i / K, k = i - y * K;
-            cp_async_8(dst + k * 16 + y, src + (int64_t)stride_y * y + k);
+            cp_async_8(dst + k * H + y, src + (int64_t)stride_y * y + k);
         }
     };
     auto load_tile = [&](const double* p, double (&x)[4][4]) {
@@ -1906,60 +1924,63 @@ __global__ void __launch_bounds__(SV_NT, 2) ccsdt_sv16_kernel(const __grid_const
     };
     if (lo >= hi) return;
     double x[4][4];  // [row][c]: xfast -> (y = row, x = c), else (x = row, y = c)
-    load_tile(plane_ptr(lo), x);
+    load_tile(unit_ptr(lo), x);
     issue_B(lo, Bs);
     cp_async_commit();
     int curA = -1;
-    for (int j = lo; j < hi; ++j) {
-        int a, o1, o2;
-        names(j, a, o1, o2);
-        if (a != curA) {
-            __syncthreads();  // every thread is done with the previous A
-            if (FAM == FAM_D1) {  // As[k][h2][h3] = v2[h3,h2,p6,k]: 16-byte copies
-                const double* src = opB + 256LL * a;
-                for (int i = tid; i < 128 * K; i += SV_NT) {
-                    const int k = i >> 7, r = 2 * (i & 127);
-                    cp_async_16(As + k * SV_PS + (r >> 4) * SV_RS + (r & 15), src + (int64_t)256 * P6 * k + r);
+    for (int u = lo; u < hi; ++u) {
+        int akey, o1, o2;
+        decode(u, akey, o1, o2);
+        if (akey != curA) {  // stage A (sign folded) for (a, f range): once or twice per CTA
+            __syncthreads();
+            const int a = akey / NFR, f0 = (akey - a * NFR) * NF;
+            if (FAM == FAM_D1) {  // As[k][fl][h3] = v2[h3, f0+fl, p6, k]: 16-byte copies
+                const double* src = opB + (int64_t)H * (f0 + (int64_t)H * a);
+                for (int i = tid; i < K * NF * (H / 2); i += NT) {
+                    const int k = i / (NF * (H / 2)), r = i - k * (NF * (H / 2));
+                    const int f = r / (H / 2), c = 2 * (r - f * (H / 2));
+                    cp_async_16(As + k * PS + f * RS + c, src + (int64_t)H * H * P6 * k + (int64_t)H * f + c);
                 }
-            } else {  // As[k][h1][h2] = t2[k,p4,h1,h2]
-                const double* src = opA + (int64_t)K * a;
-                for (int i = tid; i < 256 * K; i += SV_NT) {
-                    const int r = i / K, k = i - r * K;  // r = h1 + 16 h2
-                    cp_async_8(As + k * SV_PS + (r & 15) * SV_RS + (r >> 4), src + (int64_t)K * P4 * r + k);
+            } else {  // As[k][fl][h2] = t2[k, p4, f0+fl, h2]
+                const double* src = opA + (int64_t)K * (a + (int64_t)P4 * f0);
+                for (int i = tid; i < K * NF * H; i += NT) {
+                    const int r = i / K, k = i - r * K;  // r = fl + NF * h2
+                    const int f = r % NF, x2 = r / NF;
+                    cp_async_8(As + k * PS + f * RS + x2, src + (int64_t)K * P4 * (f + (int64_t)H * x2) + k);
                 }
             }
             cp_async_commit();
             if (sg < 0.0) {  // fold the variant's sign into A once (exact)
                 cp_async_wait_all();
                 __syncthreads();
-                for (int i = tid; i < 256 * K; i += SV_NT) {
-                    const int k = i >> 8, r = i & 255;
-                    double& v = As[k * SV_PS + (r >> 4) * SV_RS + (r & 15)];
+                for (int i = tid; i < K * NF * H; i += NT) {
+                    const int k = i / (NF * H), r = i - k * (NF * H);
+                    double& v = As[k * PS + (r / H) * RS + (r % H)];
                     v = -v;
                 }
             }
-            curA = a;
+            curA = akey;
         }
         cp_async_wait_all();
-        __syncthreads();  // B(j) landed, A staged, the other B buffer is free
-        const double* Bc = Bs + ((j - lo) & 1) * 16 * K;
-        if (j + 1 < hi) issue_B(j + 1, Bs + ((j + 1 - lo) & 1) * 16 * K);
+        __syncthreads();  // B(u) landed, A staged, the other B buffer is free
+        const double* Bc = Bs + ((u - lo) & 1) * H * K;
+        if (u + 1 < hi) issue_B(u + 1, Bs + ((u + 1 - lo) & 1) * H * K);
         cp_async_commit();
         double acc[4][4];
 #pragma unroll
         for (int r = 0; r < 4; ++r)
 #pragma unroll
             for (int c = 0; c < 4; ++c) acc[r][c] = x[r][c];
-        double* tp = plane_ptr(j);
-        if (j + 1 < hi) load_tile(plane_ptr(j + 1), x);
-        const double* Ap = As + f * SV_RS + 4 * bx;
+        double* tp = unit_ptr(u);
+        if (u + 1 < hi) load_tile(unit_ptr(u + 1), x);
+        const double* Ap = As + fl * RS + 4 * bx;
         const double* Bp = Bc + 4 * by;
 #pragma unroll 4
         for (int k = 0; k < K; ++k) {
-            const double2 a01 = *reinterpret_cast<const double2*>(Ap + k * SV_PS);
-            const double2 a23 = *reinterpret_cast<const double2*>(Ap + k * SV_PS + 2);
-            const double2 b01 = *reinterpret_cast<const double2*>(Bp + k * 16);
-            const double2 b23 = *reinterpret_cast<const double2*>(Bp + k * 16 + 2);
+            const double2 a01 = *reinterpret_cast<const double2*>(Ap + k * PS);
+            const double2 a23 = *reinterpret_cast<const double2*>(Ap + k * PS + 2);
+            const double2 b01 = *reinterpret_cast<const double2*>(Bp + k * H);
+            const double2 b23 = *reinterpret_cast<const double2*>(Bp + k * H + 2);
             const double av[4] = {a01.x, a01.y, a23.x, a23.y}, bv[4] = {b01.x, b01.y, b23.x, b23.y};
 #pragma unroll
             for (int i = 0; i < 4; ++i)
@@ -2188,29 +2209,28 @@ static int launch_ccsdt_sv16b(const CcsdtParams& P, cudaStream_t s) {
     return launch_status();
 }
 
-template <int FAM>
-static int launch_ccsdt_sv16(const CcsdtParams& P, cudaStream_t s) {
-    // register-streamed kernel by default (tile 16, back-to-back calls: 0.63-0.67 of HBM vs
-    // 0.62-0.63 for the bulk-streamed one, 0.56-0.57 for the TMA cube kernel)
-    if (getenv("BC_SV16_BULK") != nullptr) {
+template <int FAM, int H>
+static int launch_ccsdt_svs(const CcsdtParams& P, cudaStream_t s) {
+    using G = SvGeo<H>;
+    if (H == 16 && getenv("BC_SV16_BULK") != nullptr) {
         const int st = launch_ccsdt_sv16b<FAM>(P, s);
         if (st != 1) return st;
     }
     const int K = P.ext[N_K];
-    const size_t smem = ((size_t)K * SV_PS + 2 * 16 * (size_t)K) * 8;
-    const int nplanes = P.qe[3] * P.qe[4] * P.qe[5];
-    if (nplanes == 0) return BC_OK;
+    const size_t smem = ((size_t)K * G::PS + 2 * (size_t)H * K) * 8;
+    const int nunits = P.qe[3] * P.qe[4] * P.qe[5] * G::NFR;
+    if (nunits == 0) return BC_OK;
     static size_t last_smem = 0;
     static int occ = 0;
     if (smem != last_smem) {
-        cudaFuncSetAttribute(ccsdt_sv16_kernel<FAM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_sv16_kernel<FAM>, SV_NT, smem);
+        cudaFuncSetAttribute(ccsdt_svs_kernel<FAM, H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_svs_kernel<FAM, H>, G::NT, smem);
         if (occ < 1) occ = 1;
         last_smem = smem;
     }
     const int64_t cap = (int64_t)num_sms() * occ;
-    const int grid = (int)(nplanes < cap ? nplanes : cap);
-    ccsdt_sv16_kernel<FAM><<<grid, SV_NT, smem, s>>>(P, nplanes);
+    const int grid = (int)(nunits < cap ? nunits : cap);
+    ccsdt_svs_kernel<FAM, H><<<grid, G::NT, smem, s>>>(P, nunits);
     return launch_status();
 }
 
@@ -2280,10 +2300,15 @@ int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const
         const int st = launch_ccsdt_s1_stream(P, s);
         if (st != 1) return st;  // 1: factors exceed shared memory (cube kernel below)
     }
-    // one d1/d2 variant on 16^3 hole cubes: t3 streamed through registers (HBM-bound)
-    if (n == 1 && fam != FAM_S1 && ext7[N_H1] == 16 && ext7[N_H2] == 16 && ext7[N_H3] == 16 && ext7[N_K] <= 32 &&
-        getenv("BC_NO_SV16") == nullptr)
-        return fam == FAM_D1 ? launch_ccsdt_sv16<FAM_D1>(P, s) : launch_ccsdt_sv16<FAM_D2>(P, s);
+    // one d1/d2 variant on 16^3 hole volumes: t3 streamed through registers (HBM-bound).
+    // 24^3 (BC_SVS24=1) measured slower than the 24-cube TMA kernel (0.44 vs 0.51 of HBM).
+    const bool svs_h = ext7[N_H1] == 16 || (ext7[N_H1] == 24 && getenv("BC_SVS24") != nullptr);
+    if (n == 1 && fam != FAM_S1 && ext7[N_H1] == ext7[N_H2] && ext7[N_H2] == ext7[N_H3] && ext7[N_K] <= 32 &&
+        svs_h && getenv("BC_NO_SV16") == nullptr) {
+        if (ext7[N_H1] == 16)
+            return fam == FAM_D1 ? launch_ccsdt_svs<FAM_D1, 16>(P, s) : launch_ccsdt_svs<FAM_D2, 16>(P, s);
+        return fam == FAM_D1 ? launch_ccsdt_svs<FAM_D1, 24>(P, s) : launch_ccsdt_svs<FAM_D2, 24>(P, s);
+    }
     // tensor-core path: 16-cubes with 16-byte-aligned operand rows (even k, even h3 for d1).
     // It also takes hole extents the 16-cube does not divide (e.g. tile 24 = 16 + 8, ragged
     // cubes zero-filled by TMA): measured 2x faster than the 12-cube DFMA kernel at tile 24.
