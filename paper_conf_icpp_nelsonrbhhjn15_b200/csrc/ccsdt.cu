@@ -1396,7 +1396,7 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const 
     const uint32_t bar_full = base + NS * TG::STAGE_BYTES + TG::ACC * 8;
     const uint32_t bar_empty = bar_full + NS * 8;
     __shared__ double red[8];
-    __shared__ double s1v[256], s1t[16];  // s1 slices of the current variant
+    __shared__ __align__(16) double s1v[2][256], s1t[2][16];  // s1 slices, double-buffered
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
         for (int i = 0; i < NS; ++i) {
@@ -1461,10 +1461,32 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const 
     const double* ep6 = P.eps_p + P4 + P5;
     double energy = 0.0;
     int g = 0;
+    const int q0 = tid & 15, q1 = tid >> 4;
+    // s1 slice of variant v for the unit (o, qv) into buffer b: s1v[b][i2*16 + i3] =
+    // v2[O3+i3, O2+i2, p6, p5], s1t[b][i1] = t1[p4, O1+i1] (zero-filled outside the block;
+    // the sign is applied at use)
+    auto s1_issue = [&](int v, int b, const int* o, const int* qv) {
+        const int O1 = o[P.s1hpos[v][0]], O2 = o[P.s1hpos[v][1]], O3 = o[P.s1hpos[v][2]];
+        const int p4 = pick(qv, P.s1ppos[v][0]), p5 = pick(qv, P.s1ppos[v][1]), p6 = pick(qv, P.s1ppos[v][2]);
+        const int i3 = tid & 15, i2 = tid >> 4;
+        const bool ok = O3 + i3 < H3 && O2 + i2 < H2;
+        cp_async_8_zfill(&s1v[b][tid],
+                         P.s1v2[v] + (ok ? (O3 + i3) + (int64_t)H3 * ((O2 + i2) + (int64_t)H2 * (p6 + (int64_t)P6 * p5)) : 0),
+                         ok);
+        if (tid < 16) {
+            const bool okt = O1 + tid < H1;
+            cp_async_8_zfill(&s1t[b][tid], P.s1t1[v] + (okt ? p4 + (int64_t)P4 * (O1 + tid) : 0), okt);
+        }
+    };
     for (int u = blockIdx.x; u < units; u += gridDim.x) {
         int o[3], len[3], qv[3];
         decode(u, o, len, qv);
-        named_bar_sync(1, 256);  // previous unit's epilogue done with the cube
+        named_bar_sync(1, 256);  // previous unit's epilogue done with the cube and the s1 buffers
+        // the first two s1 slices land while the d1/d2 stages run
+        for (int v = 0; v < 2; ++v) {
+            if (v < P.ns1) s1_issue(v, v, o, qv);
+            cp_async_commit();
+        }
         for (int i = tid; i < BS * CST * CST; i += 256) acc_s[i] = 0.0;
         named_bar_sync(1, 256);
         double c[4][2][2];
@@ -1489,36 +1511,38 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const 
                 else tma_flush_class<FAM_D2>(acc_s, c, P.hpos[P.ecls[e]], warp, gq, tq);
             }
         }
-        named_bar_sync(1, 256);  // all d1/d2 classes flushed
-        // s1 rank-1 updates t3 += s t1[p4,h1] v2[h3,h2,p6,p5]: per variant the unit needs a
-        // 16x16 (h3,h2) slice of v2 and 16 h1 values of t1, staged in shared memory
-        const int q0 = tid & 15, q1 = tid >> 4;
+        // s1 rank-1 updates t3 += s t1[p4,h1] v2[h3,h2,p6,p5], accumulated in registers for
+        // this thread's positions (q0, q1, *) and folded into the energy epilogue (t3 is
+        // never stored, so the cube is not updated)
+        double s1acc[BS];
+#pragma unroll
+        for (int q2 = 0; q2 < BS; ++q2) s1acc[q2] = 0.0;
         for (int v = 0; v < P.ns1; ++v) {
+            const int b = v & 1;
+            cp_async_wait_n<1>();    // this thread's copies of slice v landed (v+1 may be in flight)
+            named_bar_sync(1, 256);  // everyone's copies of slice v landed
             const int hp1 = P.s1hpos[v][0], hp2 = P.s1hpos[v][1], hp3 = P.s1hpos[v][2];
-            const int p4 = pick(qv, P.s1ppos[v][0]), p5 = pick(qv, P.s1ppos[v][1]), p6 = pick(qv, P.s1ppos[v][2]);
-            {   // stage: s1v[i2*16 + i3] = v2[O3+i3, O2+i2, p6, p5]; s1t[i1] = s * t1[p4, O1+i1]
-                const int O2 = o[hp2], O3 = o[hp3], O1 = o[hp1];
-                const int i3 = tid & 15, i2 = tid >> 4;
-                const bool ok = O3 + i3 < H3 && O2 + i2 < H2;
-                s1v[tid] = ok ? __ldg(P.s1v2[v] + (O3 + i3) + (int64_t)H3 * ((O2 + i2) + (int64_t)H2 * (p6 + (int64_t)P6 * p5))) : 0.0;
-                if (tid < 16) s1t[tid] = (O1 + tid < H1) ? P.s1sign[v] * __ldg(P.s1t1[v] + p4 + (int64_t)P4 * (O1 + tid)) : 0.0;
-            }
-            named_bar_sync(1, 256);
-            // this thread's positions (q0, q1, q2 = 0..15): local hole indices by the class map
-#pragma unroll 4
+            const double sgn = P.s1sign[v];
+            const double* sv = s1v[b];
+            const double* stt = s1t[b];
+#pragma unroll
             for (int q2 = 0; q2 < BS; ++q2) {
-                const int ql0 = q0, ql1 = q1, ql2 = q2;
-                const int i1 = hp1 == 0 ? ql0 : (hp1 == 1 ? ql1 : ql2);
-                const int i2 = hp2 == 0 ? ql0 : (hp2 == 1 ? ql1 : ql2);
-                const int i3 = hp3 == 0 ? ql0 : (hp3 == 1 ? ql1 : ql2);
-                acc_s[q0 + CST * (q1 + CST * q2)] += s1t[i1] * s1v[i2 * 16 + i3];
+                const int i1 = hp1 == 0 ? q0 : (hp1 == 1 ? q1 : q2);
+                const int i2 = hp2 == 0 ? q0 : (hp2 == 1 ? q1 : q2);
+                const int i3 = hp3 == 0 ? q0 : (hp3 == 1 ? q1 : q2);
+                s1acc[q2] = fma(sgn * stt[i1], sv[i2 * 16 + i3], s1acc[q2]);
             }
-            named_bar_sync(1, 256);
+            named_bar_sync(1, 256);  // slice v consumed: its buffer takes slice v+2
+            if (v + 2 < P.ns1) s1_issue(v + 2, b, o, qv);
+            cp_async_commit();
         }
+        cp_async_wait_n<0>();
+        named_bar_sync(1, 256);  // all d1/d2 classes flushed
         // energy of every cube position this thread owns (canonical (h3,h2,h1,p6,p5,p4))
+#pragma unroll
         for (int q2 = 0; q2 < BS; ++q2) {
             if (q0 >= len[0] || q1 >= len[1] || q2 >= len[2]) continue;
-            const double t = acc_s[q0 + CST * (q1 + CST * q2)];
+            const double t = acc_s[q0 + CST * (q1 + CST * q2)] + s1acc[q2];
             const double den = ((((eh3[o[0] + q0] + eh2[o[1] + q1]) + eh1[o[2] + q2]) - ep6[qv[0]]) - ep5[qv[1]]) -
                                ep4[qv[2]];
             energy += t * t / den;
@@ -1638,7 +1662,7 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
 // ==================================================================================
 constexpr int S1S_NT = 256, S1S_U = 4;  // threads, runs in flight per thread
 #ifndef BC_S1_MINB
-#define BC_S1_MINB 1  // measured: 3 or 4 CTAs/SM (79 / 64 registers) are slower than 2 (128 registers)
+#define BC_S1_MINB 2  // measured: 2 CTAs/SM (128 registers) beat 1 (156), 3 (79) and 4 (64)
 #endif
 
 // RUN consecutive storage-position-0 values per thread (16-byte accesses when RUN = 4).
