@@ -1704,16 +1704,20 @@ __global__ void __launch_bounds__(S1S_NT, BC_S1_MINB) ccsdt_s1_stream_kernel(con
         p5 = pick(P.ppos[e][1]);
         p6 = pick(P.ppos[e][2]);
     };
-    // V factors of a plane: cp.async into buffer b
+    // V factors of a plane: cp.async into buffer b.  The plane's particle values are decoded
+    // once; this thread's first (h2, h3) is hoisted (one element per entry when H2 H3 <= NT).
+    const int vh2 = tid / (H3 > 0 ? H3 : 1), vh3 = tid - vh2 * H3;
     auto stage_v = [&](int plane, int b) {
         double* buf = s1sm + b * BUFD;
+        const int qv0 = plane % P.qe[3], qv1 = (plane / P.qe[3]) % P.qe[4], qv2 = plane / (P.qe[3] * P.qe[4]);
+        auto pick = [&](int pos) { return pos == 3 ? qv0 : (pos == 4 ? qv1 : qv2); };
         for (int e = 0; e < P.nentry; ++e) {
-            int p4, p5, p6;
-            pvals(plane, e, p4, p5, p6);
+            const int p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
             const int c = P.ecls[e], m = e - (c == 0 ? 0 : (c == 1 ? n0 : n0 + n1));
             const double* v2 = P.opB[e] + (int64_t)H3 * H2 * (p6 + (int64_t)P6 * p5);
             double* dst = buf + c * CS + m;
-            for (int i = tid; i < H2 * H3; i += S1S_NT) {
+            if (tid < H2 * H3) cp_async_8(dst + 3 * (vh2 * (H3 + 1) + vh3), v2 + tid);
+            for (int i = tid + S1S_NT; i < H2 * H3; i += S1S_NT) {
                 const int h2 = i / H3, h3 = i - h2 * H3;
                 cp_async_8(dst + 3 * (h2 * (H3 + 1) + h3), v2 + i);
             }
@@ -1783,32 +1787,21 @@ __global__ void __launch_bounds__(S1S_NT, BC_S1_MINB) ccsdt_s1_stream_kernel(con
                     } else {
                         x[u][0] = __ldcs(t3p + r);
                     }
+                } else {
+#pragma unroll
+                    for (int k = 0; k < RUN; ++k) x[u][k] = 0.0;
                 }
             }
+            // per run and class: offsets of the V row and the T entry (this run's first element)
+            int vo[S1S_U][3], to[S1S_U][3];
 #pragma unroll
             for (int u = 0; u < S1S_U; ++u) {
-                const int r = r0 + u * S1S_NT + tid;
-                if (r < nruns) {
-                    const int qq0 = q0 * RUN;
+                const int qq0 = q0 * RUN;
+                const bool ok = r0 + u * S1S_NT + tid < nruns;  // past the end: read in-range, discard
 #pragma unroll
-                    for (int c = 0; c < 3; ++c) {
-                        if (c < P.ncls) {
-                            const double* Vc = buf + c * CS + 3 * (qq0 * av[c][0] + q1 * av[c][1] + q2 * av[c][2]);
-                            const double* Tc = buf + c * CS + 3 * (VS + qq0 * at[c][0] + q1 * at[c][1] + q2 * at[c][2]);
-                            const int dv = 3 * av[c][0], dt = 3 * at[c][0];
-#pragma unroll
-                            for (int k = 0; k < RUN; ++k)
-#pragma unroll
-                                for (int m = 0; m < 3; ++m)
-                                    if (m < cnt[c]) x[u][k] = fma(Tc[k * dt + m], Vc[k * dv + m], x[u][k]);
-                        }
-                    }
-                    if constexpr (RUN == 4) {
-                        __stcs(reinterpret_cast<double2*>(t3p) + 2 * r, make_double2(x[u][0], x[u][1]));
-                        __stcs(reinterpret_cast<double2*>(t3p) + 2 * r + 1, make_double2(x[u][2], x[u][3]));
-                    } else {
-                        __stcs(t3p + r, x[u][0]);
-                    }
+                for (int c = 0; c < 3; ++c) {
+                    vo[u][c] = ok ? c * CS + 3 * (qq0 * av[c][0] + q1 * av[c][1] + q2 * av[c][2]) : 0;
+                    to[u][c] = ok ? c * CS + 3 * (VS + qq0 * at[c][0] + q1 * at[c][1] + q2 * at[c][2]) : 0;
                 }
                 q0 += d0;
                 const int c0 = q0 >= R0;
@@ -1817,6 +1810,35 @@ __global__ void __launch_bounds__(S1S_NT, BC_S1_MINB) ccsdt_s1_stream_kernel(con
                 const int c1 = q1 >= Q1;
                 q1 -= c1 ? Q1 : 0;
                 q2 += d2 + c1;
+            }
+            // entries outermost: 4 runs x RUN independent accumulation chains per entry
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                if (c < P.ncls) {
+                    const int dv = 3 * av[c][0], dt = 3 * at[c][0];
+#pragma unroll
+                    for (int m = 0; m < 3; ++m) {
+                        if (m < cnt[c]) {
+#pragma unroll
+                            for (int u = 0; u < S1S_U; ++u)
+#pragma unroll
+                                for (int k = 0; k < RUN; ++k)
+                                    x[u][k] = fma(buf[to[u][c] + k * dt + m], buf[vo[u][c] + k * dv + m], x[u][k]);
+                        }
+                    }
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < S1S_U; ++u) {
+                const int r = r0 + u * S1S_NT + tid;
+                if (r < nruns) {
+                    if constexpr (RUN == 4) {
+                        __stcs(reinterpret_cast<double2*>(t3p) + 2 * r, make_double2(x[u][0], x[u][1]));
+                        __stcs(reinterpret_cast<double2*>(t3p) + 2 * r + 1, make_double2(x[u][2], x[u][3]));
+                    } else {
+                        __stcs(t3p + r, x[u][0]);
+                    }
+                }
             }
         }
         if (t_fast && towner && nxt < nplanes) s1sm[((it + 1) & 1) * BUFD + tdst] = tsg * tnext;
