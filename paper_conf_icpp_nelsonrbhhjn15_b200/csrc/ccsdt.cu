@@ -1845,7 +1845,177 @@ __global__ void __launch_bounds__(S1S_NT, BC_S1_MINB) ccsdt_s1_stream_kernel(con
     }
 }
 
+// Equal hole extents H (16, 24): the same stream with every shape constant compile-time.
+// Per entry e (a compile-time slot): V_e [h2][h3] (row stride H+2: conflict-free 16-byte
+// reads) and T_e [h1] at fixed offsets, so every shared read is one base register plus an
+// immediate.  For s1 the name at storage position 0 is h3 or h1 (h2 always follows h3), so
+// along a run either V (4 contiguous values, T broadcast) or T (V broadcast) varies.
+template <int H>
+__global__ void __launch_bounds__(S1S_NT, 2) ccsdt_s1h_kernel(const __grid_constant__ CcsdtParams P, int nplanes) {
+    constexpr int RS = H + 2, VS = H * RS, ES = VS + H, BUFD = 9 * ES;
+    constexpr int NV = H * H * H, R0 = H / 4, NRUN = NV / 4;
+    constexpr int NB = (NRUN + S1S_NT * S1S_U - 1) / (S1S_NT * S1S_U);  // run batches per plane
+    extern __shared__ __align__(16) double s1sm[];
+    const int P4 = P.ext[N_P4], P6 = P.ext[N_P6];
+    const int tid = threadIdx.x;
+    const int ne = P.nentry;
+    // per class: V offset = qq0*av0 + q1*av1 + q2*av2, T offset = ... ; q0 is h3 (kind 0) or h1 (kind 1)
+    int av[3][3], at[3][3];
+    bool q0h1[3];
+#pragma unroll
+    for (int c = 0; c < 3; ++c) {
+        const bool ok = c < P.ncls;
+        q0h1[c] = ok && P.hpos[c][0] == 0;
+#pragma unroll
+        for (int q = 0; q < 3; ++q) {
+            at[c][q] = (ok && P.hpos[c][0] == q) ? 1 : 0;
+            av[c][q] = (ok && P.hpos[c][1] == q) ? RS : ((ok && P.hpos[c][2] == q) ? 1 : 0);
+        }
+    }
+    auto stage_v = [&](int plane, int b) {
+        const int qv0 = plane % P.qe[3], qv1 = (plane / P.qe[3]) % P.qe[4], qv2 = plane / (P.qe[3] * P.qe[4]);
+        auto pick = [&](int pos) { return pos == 3 ? qv0 : (pos == 4 ? qv1 : qv2); };
+        double* buf = s1sm + b * BUFD;
+#pragma unroll
+        for (int e = 0; e < 9; ++e) {
+            if (e < ne) {
+                const double* v2 = P.opB[e] + (int64_t)H * H * (pick(P.ppos[e][2]) + (int64_t)P6 * pick(P.ppos[e][1]));
+#pragma unroll
+                for (int i0 = 0; i0 < VS / 2; i0 += S1S_NT) {  // 16-byte chunks of the H x H slice
+                    const int i = i0 + tid;
+                    if (i < H * H / 2) {
+                        const int row = i / (H / 2), col = 2 * (i - row * (H / 2));
+                        cp_async_16(buf + e * ES + row * RS + col, v2 + row * H + col);
+                    }
+                }
+            }
+        }
+    };
+    // T (sign folded): thread t < ne*H owns T_e[h1], loaded one plane ahead into a register
+    const int te = tid / H, th1 = tid - te * H;
+    const bool towner = te < ne;
+    const double tsg = towner ? P.sign[te] : 0.0;
+    auto load_t = [&](int plane) {
+        if (!towner) return 0.0;
+        const int qv0 = plane % P.qe[3], qv1 = (plane / P.qe[3]) % P.qe[4], qv2 = plane / (P.qe[3] * P.qe[4]);
+        const int pos = P.ppos[te][0];
+        const int p4 = pos == 3 ? qv0 : (pos == 4 ? qv1 : qv2);
+        return __ldg(P.opA[te] + p4 + (int64_t)P4 * th1);
+    };
+    const int tdst = te * ES + VS + th1;
+    int it = 0;
+    if ((int)blockIdx.x < nplanes) {
+        stage_v(blockIdx.x, 0);
+        if (towner) s1sm[tdst] = tsg * load_t(blockIdx.x);
+    }
+    cp_async_commit();
+    for (int plane = blockIdx.x; plane < nplanes; plane += gridDim.x, ++it) {
+        cp_async_wait_all();
+        __syncthreads();  // this plane's factors are in place; the other buffer is free
+        const int nxt = plane + gridDim.x;
+        double tnext = 0.0;
+        if (nxt < nplanes) {
+            stage_v(nxt, (it + 1) & 1);
+            tnext = load_t(nxt);
+        }
+        cp_async_commit();
+        const double* buf = s1sm + (it & 1) * BUFD;
+        double* t3p = P.t3 + (int64_t)NV * plane;
+#pragma unroll 1
+        for (int bt = 0; bt < NB; ++bt) {
+            double x[S1S_U][4];
+            int vo[S1S_U][3], to[S1S_U][3];
+            bool ok[S1S_U];
+#pragma unroll
+            for (int u = 0; u < S1S_U; ++u) {
+                const int r = (bt * S1S_U + u) * S1S_NT + tid;
+                ok[u] = r < NRUN;
+                const int rr = ok[u] ? r : 0;
+                const int qq0 = 4 * (rr % R0), q1 = (rr / R0) % H, q2 = rr / (R0 * H);
+                if (ok[u]) {
+                    const double2 a = __ldcs(reinterpret_cast<const double2*>(t3p) + 2 * r);
+                    const double2 b = __ldcs(reinterpret_cast<const double2*>(t3p) + 2 * r + 1);
+                    x[u][0] = a.x; x[u][1] = a.y; x[u][2] = b.x; x[u][3] = b.y;
+                } else {
+                    x[u][0] = x[u][1] = x[u][2] = x[u][3] = 0.0;
+                }
+#pragma unroll
+                for (int c = 0; c < 3; ++c) {
+                    vo[u][c] = qq0 * av[c][0] + q1 * av[c][1] + q2 * av[c][2];
+                    to[u][c] = VS + qq0 * at[c][0] + q1 * at[c][1] + q2 * at[c][2];
+                }
+            }
+#pragma unroll
+            for (int e = 0; e < 9; ++e) {
+                if (e < ne) {
+                    const int c = P.ecls[e];
+                    const double* eb = buf + e * ES;
+                    const bool kind_h1 = c == 0 ? q0h1[0] : (c == 1 ? q0h1[1] : q0h1[2]);
+                    if (kind_h1) {  // run along h1: T varies, V broadcast
+#pragma unroll
+                        for (int u = 0; u < S1S_U; ++u) {
+                            const int voff = c == 0 ? vo[u][0] : (c == 1 ? vo[u][1] : vo[u][2]);
+                            const int toff = c == 0 ? to[u][0] : (c == 1 ? to[u][1] : to[u][2]);
+                            const double v = eb[voff];
+                            const double2 t01 = *reinterpret_cast<const double2*>(eb + toff);
+                            const double2 t23 = *reinterpret_cast<const double2*>(eb + toff + 2);
+                            x[u][0] = fma(t01.x, v, x[u][0]);
+                            x[u][1] = fma(t01.y, v, x[u][1]);
+                            x[u][2] = fma(t23.x, v, x[u][2]);
+                            x[u][3] = fma(t23.y, v, x[u][3]);
+                        }
+                    } else {  // run along h3: V varies, T broadcast
+#pragma unroll
+                        for (int u = 0; u < S1S_U; ++u) {
+                            const int voff = c == 0 ? vo[u][0] : (c == 1 ? vo[u][1] : vo[u][2]);
+                            const int toff = c == 0 ? to[u][0] : (c == 1 ? to[u][1] : to[u][2]);
+                            const double t = eb[toff];
+                            const double2 v01 = *reinterpret_cast<const double2*>(eb + voff);
+                            const double2 v23 = *reinterpret_cast<const double2*>(eb + voff + 2);
+                            x[u][0] = fma(t, v01.x, x[u][0]);
+                            x[u][1] = fma(t, v01.y, x[u][1]);
+                            x[u][2] = fma(t, v23.x, x[u][2]);
+                            x[u][3] = fma(t, v23.y, x[u][3]);
+                        }
+                    }
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < S1S_U; ++u) {
+                const int r = (bt * S1S_U + u) * S1S_NT + tid;
+                if (ok[u]) {
+                    __stcs(reinterpret_cast<double2*>(t3p) + 2 * r, make_double2(x[u][0], x[u][1]));
+                    __stcs(reinterpret_cast<double2*>(t3p) + 2 * r + 1, make_double2(x[u][2], x[u][3]));
+                }
+            }
+        }
+        if (towner && nxt < nplanes) s1sm[((it + 1) & 1) * BUFD + tdst] = tsg * tnext;
+    }
+}
+
+template <int H>
+static int launch_ccsdt_s1h(const CcsdtParams& P, cudaStream_t s) {
+    constexpr size_t smem = 2 * 9 * (size_t)(H * (H + 2) + H) * 8;
+    const int nplanes = P.qe[3] * P.qe[4] * P.qe[5];
+    if (nplanes == 0) return BC_OK;
+    static int occ = 0;
+    if (occ == 0) {
+        cudaFuncSetAttribute(ccsdt_s1h_kernel<H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_s1h_kernel<H>, S1S_NT, smem);
+        if (occ < 1) occ = 1;
+    }
+    const int64_t cap = (int64_t)num_sms() * occ;
+    const int grid = (int)(nplanes < cap ? nplanes : cap);
+    ccsdt_s1h_kernel<H><<<grid, S1S_NT, smem, s>>>(P, nplanes);
+    return launch_status();
+}
+
 static int launch_ccsdt_s1_stream(const CcsdtParams& P, cudaStream_t s) {
+    const int H = P.ext[N_H1];
+    if (H == P.ext[N_H2] && H == P.ext[N_H3] && getenv("BC_S1_GENERIC") == nullptr) {
+        if (H == 16) return launch_ccsdt_s1h<16>(P, s);
+        if (H == 24) return launch_ccsdt_s1h<24>(P, s);
+    }
     const size_t smem = 2 * ((size_t)P.ncls * 3 * (P.ext[N_H2] * (P.ext[N_H3] + 1) + P.ext[N_H1])) * 8;
     if (smem > 200 * 1024) return 1;
     const int nplanes = P.qe[3] * P.qe[4] * P.qe[5];

@@ -343,6 +343,9 @@ enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
 #ifndef BC_E13
 #define BC_E13 3
 #endif
+#ifndef AXE_PB
+#define AXE_PB 4  // ax_e: points per thread whose 6 geometric factors are loaded together
+#endif
 #ifndef BC_SF2_UNROLL
 #define BC_SF2_UNROLL 1
 #endif
@@ -656,17 +659,30 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
         apply_lines<P1, P1, 2, R, NT>(bR, opD, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
         __syncthreads();
         const int total = ne * G::NPTS;
-        for (int f = threadIdx.x; f < total; f += NT) {  // G[e][c][q]
-            const int e = f / G::NPTS;
-            const int q = f - e * G::NPTS;
-            const T* gp = Gm + (e0 + e) * 6 * (int64_t)G::NPTS + q;
-            const T g0 = __ldcs(gp), g1 = __ldcs(gp + G::NPTS), g2 = __ldcs(gp + 2 * G::NPTS),
-                    g3 = __ldcs(gp + 3 * G::NPTS), g4 = __ldcs(gp + 4 * G::NPTS), g5 = __ldcs(gp + 5 * G::NPTS);
-            const int si = smem_index<P1, P1, T>(f);
-            const T r = bR[si], s = bS[si], t = bT[si];
-            bR[si] = (g0 * r + g1 * s) + g2 * t;
-            bS[si] = (g1 * r + g3 * s) + g4 * t;
-            bT[si] = (g2 * r + g4 * s) + g5 * t;
+        // G[e][c][q]: AXE_PB points per thread per batch, all 6*AXE_PB loads issued before use
+        constexpr int PB = AXE_PB;
+        for (int f0 = threadIdx.x; f0 < total; f0 += PB * NT) {
+            T gv[PB][6];
+#pragma unroll
+            for (int b = 0; b < PB; ++b) {
+                const int f = f0 + b * NT;
+                const int fc = f < total ? f : f0;
+                const int e = fc / G::NPTS;
+                const T* gp = Gm + (e0 + e) * 6 * (int64_t)G::NPTS + (fc - e * G::NPTS);
+#pragma unroll
+                for (int c = 0; c < 6; ++c) gv[b][c] = __ldcs(gp + c * G::NPTS);
+            }
+#pragma unroll
+            for (int b = 0; b < PB; ++b) {
+                const int f = f0 + b * NT;
+                if (f < total) {
+                    const int si = smem_index<P1, P1, T>(f);
+                    const T r = bR[si], s = bS[si], t = bT[si];
+                    bR[si] = (gv[b][0] * r + gv[b][1] * s) + gv[b][2] * t;
+                    bS[si] = (gv[b][1] * r + gv[b][3] * s) + gv[b][4] * t;
+                    bT[si] = (gv[b][2] * r + gv[b][4] * s) + gv[b][5] * t;
+                }
+            }
         }
         __syncthreads();
         apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });

@@ -55,7 +55,8 @@ def test_single_variant_integer_bitwise(bc, family, ext):
 
 
 @pytest.mark.parametrize("family", ["d1", "d2", "s1"])
-@pytest.mark.parametrize("ext", [(3, 4, 5, 6, 2, 7, 3), (12, 12, 12, 7, 7, 7, 21), (5, 5, 5, 3, 3, 3, 40)])
+@pytest.mark.parametrize("ext", [(3, 4, 5, 6, 2, 7, 3), (12, 12, 12, 7, 7, 7, 21), (5, 5, 5, 3, 3, 3, 40),
+                                 (16, 16, 16, 3, 3, 3, 4), (24, 24, 24, 2, 2, 2, 4)])
 def test_fused_integer_bitwise(bc, family, ext):
     na, nb = sizes(family, ext)
     t3 = syn.tensor(10, (n3(ext),), kind=syn.KIND_INT)
