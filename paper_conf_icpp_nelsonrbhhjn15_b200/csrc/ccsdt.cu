@@ -340,10 +340,6 @@ __device__ __forceinline__ void cp_async_16_zfill(void* dst, const void* src, bo
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(smem_u32(dst)), "l"(src),
                  "r"(valid ? 16 : 0));
 }
-template <int N>
-__device__ __forceinline__ void cp_async_wait_n() {
-    asm volatile("cp.async.wait_group %0;\n" ::"n"(N));
-}
 
 template <int FAM>
 __global__ void __launch_bounds__(256) ccsdt_mma_kernel(const CcsdtParams P) {

@@ -60,6 +60,10 @@ __device__ __forceinline__ void cp_async_4(void* dst, const void* src) {
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait_n() {  // at most N of this thread's groups pending
+    asm volatile("cp.async.wait_group %0;\n" ::"n"(N));
+}
 
 template <typename T>
 __device__ __forceinline__ void cp_async_elem(T* dst, const T* src) {

@@ -594,17 +594,23 @@ local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __re
         const int nlines = ne * P1 * P1;
         const int64_t gbase = e0 * G::NPTS;
         __syncthreads();  // previous group fully consumed
+        // one cp.async group per field: the r stage starts as soon as ur has landed while us
+        // and ut are still in flight
         T* bR = load_group_async<P1, P1, T, NT>(bR0, ur + gbase, ne);
+        cp_async_commit();
         T* bS = load_group_async<P1, P1, T, NT>(bS0, us + gbase, ne);
+        cp_async_commit();
         T* bT = load_group_async<P1, P1, T, NT>(bT0, ut + gbase, ne);
         cp_async_commit();
-        cp_async_wait_all();
+        cp_async_wait_n<2>();
         __syncthreads();
         apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
+        cp_async_wait_n<1>();
         __syncthreads();
         apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines, [&](int, int base, int k, T v) {
             bS[base + k * G::RS] = bR[base + k * G::RS] + v;
         });
+        cp_async_wait_n<0>();
         __syncthreads();
         apply_lines<P1, P1, 0, R, NT>(bT, opT, nlines, [&](int L, int base, int k, T v) {
             st_cs(U + gbase + Line<P1, P1, 0, T>::gofs(L, k), bS[base + k * G::PS] + v);
