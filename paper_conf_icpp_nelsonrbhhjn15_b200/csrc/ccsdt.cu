@@ -1558,6 +1558,250 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const 
     }
 }
 
+// ---- f4 on exact 24-cubes (hole extents 24, the tile-24 block): the tile-24 DMMA scheme of
+// ccsdt_tma24_kernel with d1 and d2 entries mixed in one TMA ring (2 stages, so that the
+// 24-cube, the ring and the double-buffered s1 slices fit one SM), the cube zeroed per unit
+// instead of seeded, s1 applied to the cube, and the energy epilogue instead of the store.
+// (The 16-cube f4 kernel covers 24 as 16 + 8: 2.37x the useful volume.)
+struct Trip24Geo {
+    static constexpr int BS = 24, KC = 8, NS = 2, NCW = 8, NT = (NCW + 1) * 32, NCT = NCW * 32;
+    static constexpr int STAGE_BYTES = Tma24Geo::STAGE_BYTES, A_BYTES = Tma24Geo::A_BYTES;
+    static constexpr int C1 = Tma24Geo::C1, C2 = Tma24Geo::C2, ACC = Tma24Geo::ACC;
+    static constexpr size_t SMEM = 1024 + (size_t)NS * STAGE_BYTES + (size_t)ACC * 8 + 2 * NS * 8;
+};
+
+// consumer: one KC = 8 stage of the 24-cube DMMA for family FE (see ccsdt_tma24_kernel)
+template <int FE>
+__device__ __forceinline__ void t24_consume(const unsigned char* A, const unsigned char* B, uint32_t smask,
+                                            double (&c)[9][3][2], int warp, int gq, int tq) {
+    constexpr int KC = Trip24Geo::KC;
+    double bf[KC / 4][3], af[KC / 4][9];
+#pragma unroll
+    for (int ks = 0; ks < KC / 4; ++ks) {
+        const unsigned char* Bk = B + swz64(perm64(gq), 4 * ks + tq);
+        const unsigned char* Ak = (FE == FAM_D1) ? A + ((4 * ks + tq) * 576 + 72 * warp + gq) * 8
+                                                 : A + 9 * warp * 512 + swz64(perm64(gq), 4 * ks + tq);
+#pragma unroll
+        for (int ni = 0; ni < 3; ++ni) bf[ks][ni] = lds64(Bk + ni * 512);
+#pragma unroll
+        for (int mi = 0; mi < 9; ++mi)
+            af[ks][mi] = lds64(Ak + ((FE == FAM_D1) ? ((mi / 3) * 24 + 8 * (mi % 3)) * 8 : mi * 512));
+    }
+#pragma unroll
+    for (int ks = 0; ks < KC / 4; ++ks)
+#pragma unroll
+        for (int ni = 0; ni < 3; ++ni) bf[ks][ni] = flip_sign(bf[ks][ni], smask);
+#pragma unroll
+    for (int ks = 0; ks < KC / 4; ++ks)
+#pragma unroll
+        for (int mi = 0; mi < 9; ++mi)
+#pragma unroll
+            for (int ni = 0; ni < 3; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[ks][mi], bf[ks][ni]);
+}
+
+// consumer: add a class's register tile into the 24-cube at its permuted positions, clear it
+template <int FE>
+__device__ __forceinline__ void t24_flush(double* acc_s, double (&c)[9][3][2], const int* hp, int warp, int gq,
+                                          int tq) {
+    constexpr int C1 = Trip24Geo::C1, C2 = Trip24Geo::C2;
+    const int s1 = hp[0] == 0 ? 1 : (hp[0] == 1 ? C1 : C2);
+    const int s2 = hp[1] == 0 ? 1 : (hp[1] == 1 ? C1 : C2);
+    const int s3 = hp[2] == 0 ? 1 : (hp[2] == 1 ? C1 : C2);
+    const int slo = (FE == FAM_D1) ? s3 : s1;
+    const int sth = (FE == FAM_D1) ? s1 : s3;
+#pragma unroll
+    for (int mi = 0; mi < 9; ++mi) {
+        const int h2 = 3 * warp + mi / 3;
+        const int lo = 8 * (mi % 3) + ((FE == FAM_D1) ? gq : perm64(gq));
+        double* row = acc_s + lo * slo + h2 * s2;
+#pragma unroll
+        for (int ni = 0; ni < 3; ++ni)
+#pragma unroll
+            for (int j = 0; j < 2; ++j) {
+                row[(8 * ni + perm64(2 * tq + j)) * sth] += c[mi][ni][j];
+                c[mi][ni][j] = 0.0;
+            }
+    }
+}
+
+__global__ void __launch_bounds__(Trip24Geo::NT, 1) ccsdt_triples24_kernel(const __grid_constant__ TripParams P,
+                                                                          const __grid_constant__ TripMaps M,
+                                                                          int units) {
+    using TG = Trip24Geo;
+    constexpr int BS = TG::BS, KC = TG::KC, NS = TG::NS, NCT = TG::NCT, C1 = TG::C1, C2 = TG::C2;
+    extern __shared__ unsigned char smem_raw[];
+    const uint32_t raw = smem_u32(smem_raw);
+    const uint32_t base = (raw + 1023) & ~1023u;
+    unsigned char* gbase = smem_raw + (base - raw);
+    double* acc_s = reinterpret_cast<double*>(gbase + NS * TG::STAGE_BYTES);
+    const uint32_t bar_full = base + NS * TG::STAGE_BYTES + TG::ACC * 8;
+    const uint32_t bar_empty = bar_full + NS * 8;
+    __shared__ double red[8];
+    __shared__ __align__(16) double s1v[2][576], s1t[2][24];  // s1 slices, double-buffered
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < NS; ++i) {
+            mbar_init(bar_full + 8 * i, 1);
+            mbar_init(bar_empty + 8 * i, TG::NCW);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    __syncthreads();
+    const int K = P.ext[N_K];
+    const int nchunk = (K + KC - 1) / KC;
+    const int nstage = P.nentry * nchunk;
+    auto decode = [&](int plane, int* qv) {  // one exact cube per particle plane
+        qv[0] = plane % P.qe[3];
+        qv[1] = (plane / P.qe[3]) % P.qe[4];
+        qv[2] = plane / (P.qe[3] * P.qe[4]);
+    };
+    auto pick = [](const int* qv, int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
+
+    if (warp == TG::NCW) {
+        int g = 0;
+        for (int u = blockIdx.x; u < units; u += gridDim.x) {
+            int qv[3];
+            decode(u, qv);
+            for (int st = 0; st < nstage; ++st, ++g) {
+                const int slot = g % NS;
+                const uint32_t full = bar_full + 8 * slot;
+                if (lane == 0) {
+                    mbar_wait(bar_empty + 8 * slot, ((g / NS) & 1) ^ 1);
+                    mbar_expect_tx(full, TG::STAGE_BYTES);
+                }
+                __syncwarp();
+                const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+                const int p4 = pick(qv, P.ppos[e][0]), p5 = pick(qv, P.ppos[e][1]), p6 = pick(qv, P.ppos[e][2]);
+                const uint32_t A = base + slot * TG::STAGE_BYTES;
+                const uint32_t B = A + TG::A_BYTES;
+                if (P.efam[e] == FAM_D1) {  // one cube: every hole offset is 0
+                    if (lane == 0) tma_load_4d(A, &M.a[e], 0, 0, p6, k0, full);
+                    if (lane == 1) tma_load_4d(B, &M.b[e], k0, p4, p5, 0, full);
+                } else {
+                    if (lane == 0) tma_load_4d(A, &M.a[e], k0, p4, 0, 0, full);
+                    if (lane == 1) tma_load_4d(B, &M.b[e], k0, 0, p6, p5, full);
+                }
+            }
+        }
+        return;
+    }
+
+    // ==================================== consumers (warps 0..7)
+    const int gq = lane >> 2, tq = lane & 3;
+    const int tid = threadIdx.x;
+    const int P4 = P.ext[N_P4], P6 = P.ext[N_P6];
+    const double* eh1 = P.eps_h;
+    const double* eh2 = P.eps_h + BS;
+    const double* eh3 = P.eps_h + 2 * BS;
+    const double* ep4 = P.eps_p;
+    const double* ep5 = P.eps_p + P4;
+    const double* ep6 = P.eps_p + 2 * P4;
+    auto s1_issue = [&](int v, int b, const int* qv) {
+        const int p4 = pick(qv, P.s1ppos[v][0]), p5 = pick(qv, P.s1ppos[v][1]), p6 = pick(qv, P.s1ppos[v][2]);
+        const double* src = P.s1v2[v] + (int64_t)BS * BS * (p6 + (int64_t)P6 * p5);  // [h3 + 24 h2]
+        for (int i = tid; i < 288; i += NCT) cp_async_16(&s1v[b][2 * i], src + 2 * i);
+        if (tid < BS) cp_async_8(&s1t[b][tid], P.s1t1[v] + p4 + (int64_t)P4 * tid);
+    };
+    double energy = 0.0;
+    int g = 0;
+    for (int u = blockIdx.x; u < units; u += gridDim.x) {
+        int qv[3];
+        decode(u, qv);
+        named_bar_sync(1, NCT);  // previous unit's epilogue done with the cube and s1 buffers
+        for (int v = 0; v < 2; ++v) {
+            if (v < P.ns1) s1_issue(v, v, qv);
+            cp_async_commit();
+        }
+        for (int i = tid; i < TG::ACC; i += NCT) acc_s[i] = 0.0;
+        named_bar_sync(1, NCT);
+        double c[9][3][2];
+#pragma unroll
+        for (int mi = 0; mi < 9; ++mi)
+#pragma unroll
+            for (int ni = 0; ni < 3; ++ni) c[mi][ni][0] = c[mi][ni][1] = 0.0;
+        int e = 0, kc_i = 0, cls_stages = 0;
+        for (int st = 0; st < nstage; ++st, ++g) {
+            ++cls_stages;
+            const int slot = g % NS;
+            mbar_wait(bar_full + 8 * slot, (g / NS) & 1);
+            const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
+            const unsigned char* B = A + TG::A_BYTES;
+            const bool d1 = P.efam[e] == FAM_D1;
+            if (d1) t24_consume<FAM_D1>(A, B, P.smask[e], c, warp, gq, tq);
+            else t24_consume<FAM_D2>(A, B, P.smask[e], c, warp, gq, tq);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
+            const bool last_chunk = (++kc_i == nchunk);
+            const int e_cur = e;
+            if (last_chunk) {
+                kc_i = 0;
+                ++e;
+            }
+            const bool class_end = last_chunk && (e == P.nentry || P.ecls[e] != P.ecls[e_cur]);
+            if (class_end) {
+                // as in ccsdt_tma24_kernel: a barrier only when the ending class spans <= NS
+                // stages (otherwise no warp can be flushing the previous class)
+                if (cls_stages <= NS) named_bar_sync(1, NCT);
+                cls_stages = 0;
+                if (d1) t24_flush<FAM_D1>(acc_s, c, P.hpos[P.ecls[e_cur]], warp, gq, tq);
+                else t24_flush<FAM_D2>(acc_s, c, P.hpos[P.ecls[e_cur]], warp, gq, tq);
+            }
+        }
+        // s1 rank-1 updates into the cube, one variant at a time (slices double-buffered)
+        for (int v = 0; v < P.ns1; ++v) {
+            const int b = v & 1;
+            cp_async_wait_n<1>();
+            named_bar_sync(1, NCT);  // slice v landed; all d1/d2 flushes are done
+            const int hp1 = P.s1hpos[v][0], hp2 = P.s1hpos[v][1], hp3 = P.s1hpos[v][2];
+            const double sgn = P.s1sign[v];
+            // (q0, q1) rows of 24 q2 values: the name-to-coordinate selects are per row, the
+            // q2 steps are strides
+            for (int i = tid; i < BS * BS; i += NCT) {
+                const int q1 = i / BS, q0 = i - q1 * BS;
+                // name index = a + b q2 for each of h1, h2, h3
+                const int a1 = hp1 == 0 ? q0 : (hp1 == 1 ? q1 : 0), b1 = hp1 == 2;
+                const int a2 = hp2 == 0 ? q0 : (hp2 == 1 ? q1 : 0), b2 = hp2 == 2;
+                const int a3 = hp3 == 0 ? q0 : (hp3 == 1 ? q1 : 0), b3 = hp3 == 2;
+                const double* tp = s1t[b] + a1;
+                const double* vp = s1v[b] + a2 * BS + a3;
+                const int dt = b1, dv = b2 * BS + b3;
+                double* xp = acc_s + q0 + C1 * q1;
+#pragma unroll 8
+                for (int q2 = 0; q2 < BS; ++q2) xp[C2 * q2] = fma(sgn * tp[dt * q2], vp[dv * q2], xp[C2 * q2]);
+            }
+            named_bar_sync(1, NCT);  // slice v consumed: its buffer takes slice v+2
+            if (v + 2 < P.ns1) s1_issue(v + 2, b, qv);
+            cp_async_commit();
+        }
+        cp_async_wait_n<0>();
+        named_bar_sync(1, NCT);  // all updates of the cube are done
+        // energy over the canonical (h3,h2,h1,p6,p5,p4) positions: (q0,q1,q2) = (h3,h2,h1)
+        const double e6 = ep6[qv[0]], e5 = ep5[qv[1]], e4 = ep4[qv[2]];
+        for (int i = tid; i < BS * BS; i += NCT) {
+            const int q1 = i / BS, q0 = i - q1 * BS;
+            const double h32 = eh3[q0] + eh2[q1];
+            const double* xp = acc_s + q0 + C1 * q1;
+#pragma unroll 4
+            for (int q2 = 0; q2 < BS; ++q2) {
+                const double t = xp[C2 * q2];
+                const double den = (((h32 + eh1[q2]) - e6) - e5) - e4;
+                energy += t * t / den;
+                if (P.dump)
+                    P.dump[q0 + (int64_t)BS * (q1 + (int64_t)BS * (q2 + (int64_t)BS * (qv[0] + (int64_t)P.qe[3] *
+                           (qv[1] + (int64_t)P.qe[4] * qv[2]))))] = t;
+            }
+        }
+    }
+    for (int off = 16; off > 0; off >>= 1) energy += __shfl_xor_sync(0xffffffffu, energy, off);
+    if (lane == 0) red[warp] = energy;
+    named_bar_sync(1, NCT);
+    if (tid == 0) {
+        double sum = 0.0;
+        for (int w = 0; w < TG::NCW; ++w) sum += red[w];
+        P.ws[8 + blockIdx.x] = sum;
+    }
+}
+
 static double* g_triples_dump = nullptr;  // debug only
 void set_triples_dump(double* p) { g_triples_dump = p; }
 
@@ -1575,6 +1819,8 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
     for (int q = 0; q < 3; ++q) P.qe[q] = H;
     for (int q = 3; q < 6; ++q) P.qe[q] = PP;
     for (int q = 0; q < 3; ++q) P.ncube[q] = (H + 15) / 16;
+    // exact 24-cubes (tile 24): the 24-cube kernel (BC_NO_TRIP24: the 16-cube one)
+    const bool c24 = H == 24 && K % 2 == 0 && getenv("BC_NO_TRIP24") == nullptr;
     P.eps_h = eps_h;
     P.eps_p = eps_p;
     P.ws = ws;
@@ -1598,7 +1844,20 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
                 P.ecls[n] = ncls;
                 P.smask[n] = vi.sign < 0 ? 0x80000000u : 0u;
                 bool ok;
-                if (fam == FAM_D1) {
+                if (c24) {  // the tile-24 boxes of ccsdt_tma24_kernel
+                    constexpr int KC24 = Trip24Geo::KC;
+                    if (fam == FAM_D1) {
+                        const int da[4] = {H, H, PP, K}, ba[4] = {24, 24, 1, KC24};
+                        const int db[4] = {K, PP, PP, H}, bb[4] = {KC24, 1, 1, 24};
+                        ok = encode_4d_sw(&M.a[n], vB[f][v - 1], da, ba, CU_TENSOR_MAP_SWIZZLE_NONE) &&
+                             encode_4d_sw(&M.b[n], tA[f][v - 1], db, bb, CU_TENSOR_MAP_SWIZZLE_64B);
+                    } else {
+                        const int da[4] = {K, PP, H, H}, ba[4] = {KC24, 1, 24, 24};
+                        const int db[4] = {K, H, PP, PP}, bb[4] = {KC24, 24, 1, 1};
+                        ok = encode_4d_sw(&M.a[n], tA[f][v - 1], da, ba, CU_TENSOR_MAP_SWIZZLE_64B) &&
+                             encode_4d_sw(&M.b[n], vB[f][v - 1], db, bb, CU_TENSOR_MAP_SWIZZLE_64B);
+                    }
+                } else if (fam == FAM_D1) {
                     const int da[4] = {H, H, PP, K};
                     const int db[4] = {K, PP, PP, H}, bb[4] = {TmaGeo::KC, 1, 1, 16};
                     ok = encode_d1_a16(&M.a[n], vB[f][v - 1], da) &&
@@ -1628,6 +1887,22 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
         ++ns;
     }
     P.ns1 = ns;
+    if (c24) {
+        static int occ24 = 0;
+        if (occ24 == 0) {
+            cudaFuncSetAttribute(ccsdt_triples24_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Trip24Geo::SMEM);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ24, ccsdt_triples24_kernel, Trip24Geo::NT, Trip24Geo::SMEM);
+            if (occ24 < 1) occ24 = 1;
+        }
+        const int units24 = PP * PP * PP;
+        int grid = num_sms() * occ24;
+        if (grid > units24) grid = units24;
+        if (grid > CHECK_MAX_PARTIALS) grid = CHECK_MAX_PARTIALS;
+        ccsdt_triples24_kernel<<<grid, Trip24Geo::NT, Trip24Geo::SMEM, s>>>(P, M, units24);
+        const int st = launch_status();
+        if (st) return st;
+        return run_check_finalize(grid, ws, s);
+    }
     static int occ = 0;
     if (occ == 0) {
         cudaFuncSetAttribute(ccsdt_triples_energy_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TmaGeo::SMEM);

@@ -130,7 +130,9 @@ def test_energy_check(bc):
     assert abs(got - ref) <= 1e-12 * abs(ref)
 
 
-@pytest.mark.parametrize("ext", [(16,) * 7, (20, 20, 20, 4, 4, 4, 6)])
+# (24, ...) takes the exact-24-cube kernel (ccsdt_triples24_kernel): k = 8 (one chunk) and
+# k = 10 (a ragged second chunk, zero-filled by TMA)
+@pytest.mark.parametrize("ext", [(16,) * 7, (20, 20, 20, 4, 4, 4, 6), (24, 24, 24, 2, 2, 2, 8), (24, 24, 24, 2, 2, 2, 10)])
 @pytest.mark.parametrize("mask", ["all", "some"])
 def test_triples_energy_f4(bc, ext, mask):
     """f4: all 27 variants fused, t3 never stored, energy epilogue == oracle energy of the t3
