@@ -142,13 +142,15 @@ struct Line {
 // 16-byte broadcast operator load feeds 2R FMAs and there are P1*R independent FMA
 // chains per thread.  All reads of a line precede the writes of that line and every
 // line is read by exactly one thread, so `out` may overwrite the line in place.
-template <int P1, int NA, int AXIS, int R, int NT, bool SWP, typename T, typename Out>
+template <int P1, int NA, int AXIS, int R, int NT, bool SWP, int UNR, typename T, typename Out>
 __device__ __forceinline__ void apply_lines_w(const T* in, const T* opT, int nlines, Out out);
 
 template <int P1, int NA, int AXIS, int R, int NT, typename T, typename Out, int UNR = BC_NUNROLL>
 __device__ __forceinline__ void apply_lines(const T* in, const T* opT, int nlines, Out out) {
-    if constexpr (BC_WCHUNK && UNR == 1) {
-        apply_lines_w<P1, NA, AXIS, R, NT, (bool)BC_SWP>(in, opT, nlines, out);
+    // fully unrolled chunks spill beyond P1 = 12 (ptxas, 255 registers at P1 = 13): those
+    // keep the lane-strided loop
+    if constexpr (BC_WCHUNK && (UNR == 1 || P1 <= 12)) {
+        apply_lines_w<P1, NA, AXIS, R, NT, (bool)BC_SWP && UNR == 1, UNR>(in, opT, nlines, out);
         return;
     }
     using G = Geo<P1, NA, T>;
@@ -202,7 +204,7 @@ __device__ __forceinline__ void apply_lines(const T* in, const T* opT, int nline
 // are computed on the chunk's first line (always valid) and not stored.  SWP: the operands of step n+1 are loaded
 // while step n's FMAs run (two register sets, ping-pong), hiding the shared-memory latency
 // that otherwise stalls every step's first FMA.
-template <int P1, int NA, int AXIS, int RR, bool SWP, typename T, typename Out>
+template <int P1, int NA, int AXIS, int RR, bool SWP, int UNR, typename T, typename Out>
 __device__ __forceinline__ void lines_chunk(const T* in, const T* opT, int L0, int nlines, Out& out) {
     using G = Geo<P1, NA, T>;
     using LN = Line<P1, NA, AXIS, T>;
@@ -253,7 +255,7 @@ __device__ __forceinline__ void lines_chunk(const T* in, const T* opT, int L0, i
         }
         if constexpr (P1 & 1) fmas(xa, oa, za);
     } else {
-#pragma unroll 1
+#pragma unroll UNR
         for (int n = 0; n < P1; ++n) {
             T x[RR], z = T(0);
             P2 o[KP];
@@ -273,19 +275,19 @@ __device__ __forceinline__ void lines_chunk(const T* in, const T* opT, int L0, i
 // into chunks of 32*R (lane-interleaved, so every strided line read stays conflict-free);
 // chunks go round-robin to the warps and the ragged last chunk runs with
 // RR = ceil(rest/32) <= R lines per lane, so no warp computes duplicate lines.
-template <int P1, int NA, int AXIS, int R, int NT, bool SWP, typename T, typename Out>
+template <int P1, int NA, int AXIS, int R, int NT, bool SWP, int UNR, typename T, typename Out>
 __device__ __forceinline__ void apply_lines_w(const T* in, const T* opT, int nlines, Out out) {
     constexpr int NW = NT / 32, CH = 32 * R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nfull = nlines / CH;
-    for (int c = warp; c < nfull; c += NW) lines_chunk<P1, NA, AXIS, R, SWP>(in, opT, c * CH + lane, nlines, out);
+    for (int c = warp; c < nfull; c += NW) lines_chunk<P1, NA, AXIS, R, SWP, UNR>(in, opT, c * CH + lane, nlines, out);
     const int rest = nlines - nfull * CH;
     if (rest > 0 && warp == nfull % NW) {
         const int L0 = nfull * CH + lane, rr = (rest + 31) >> 5;
-        if constexpr (R >= 4) if (rr == 4) { lines_chunk<P1, NA, AXIS, 4, SWP>(in, opT, L0, nlines, out); return; }
-        if constexpr (R >= 3) if (rr == 3) { lines_chunk<P1, NA, AXIS, (R >= 3 ? 3 : 1), SWP>(in, opT, L0, nlines, out); return; }
-        if constexpr (R >= 2) if (rr == 2) { lines_chunk<P1, NA, AXIS, (R >= 2 ? 2 : 1), SWP>(in, opT, L0, nlines, out); return; }
-        lines_chunk<P1, NA, AXIS, 1, SWP>(in, opT, L0, nlines, out);
+        if constexpr (R >= 4) if (rr == 4) { lines_chunk<P1, NA, AXIS, 4, SWP, UNR>(in, opT, L0, nlines, out); return; }
+        if constexpr (R >= 3) if (rr == 3) { lines_chunk<P1, NA, AXIS, (R >= 3 ? 3 : 1), SWP, UNR>(in, opT, L0, nlines, out); return; }
+        if constexpr (R >= 2) if (rr == 2) { lines_chunk<P1, NA, AXIS, (R >= 2 ? 2 : 1), SWP, UNR>(in, opT, L0, nlines, out); return; }
+        lines_chunk<P1, NA, AXIS, 1, SWP, UNR>(in, opT, L0, nlines, out);
     }
 }
 
