@@ -336,6 +336,10 @@ enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
 #ifndef BC_BIG_R
 #define BC_BIG_R 4
 #endif
+#ifndef BC_SMALL_R
+#define BC_SMALL_R 3  // sumfact3d lines per thread at P1 < 10 (measured: p=4 0.57 -> 0.65, p=5 0.56 -> 0.62,
+                      // p=8 0.47 -> 0.53 of HBM vs R = 2; local_grad3 stays at R = 2)
+#endif
 #ifndef BC_BIG_KB
 #define BC_BIG_KB 54
 #endif
@@ -356,7 +360,8 @@ struct SpecTable {
     static constexpr bool BIG = P1 >= 10;
     static constexpr bool SF3LG3 = KIND == K_SF3 || KIND == K_LG3;
     static constexpr bool MID = P1 == 12;  // sumfact3d / local_grad3: R = 3, 36 KiB (measured)
-    static constexpr int R = BIG ? (SF3LG3 ? (MID ? 3 : BC_BIG_R) : (KIND == K_SF2 ? 3 : 2)) : 2;
+    static constexpr int R = BIG ? (SF3LG3 ? (MID ? 3 : BC_BIG_R) : (KIND == K_SF2 ? 3 : 2))
+                                 : (KIND == K_SF3 ? BC_SMALL_R : 2);
     static constexpr int BUF_KB = BIG ? (SF3LG3 ? (MID ? 36 : BC_BIG_KB) : 18) : (KIND == K_LG3 ? 36 : 18);
     static constexpr bool PREFETCH = !(BIG && SF3LG3) || BC_BIG_PF;
     // forced elements per group (0: derived from BUF_KB): P1 = 13: 3 x 169 = 507 lines on
