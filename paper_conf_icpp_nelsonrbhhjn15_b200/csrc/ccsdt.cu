@@ -2377,29 +2377,48 @@ __global__ void __launch_bounds__(SvGeo<H>::NT, SvGeo<H>::MINB) ccsdt_svs_kernel
     const double* __restrict__ opB = P.opB[0];  // v2
     const int lo = (int)((int64_t)nunits * blockIdx.x / gridDim.x);
     const int hi = (int)((int64_t)nunits * (blockIdx.x + 1) / gridDim.x);
-    // unit u -> (a, fr, o1, o2), a = the A name (d1 p6, d2 p4) slowest
-    auto decode = [&](int u, int& akey, int& o1, int& o2) {
-        akey = u / (PO1 * PO2);  // a * NFR + fr
-        const int r = u - akey * (PO1 * PO2);
-        o1 = r / PO2;
-        o2 = r - o1 * PO2;
+    // unit u -> (akey = a * NFR + fr, o1, o2), a = the A name (d1 p6, d2 p4) slowest; decoded
+    // once per CTA and then advanced by carries (no divisions per unit)
+    struct UnitId { int akey, o1, o2; };
+    auto decode = [&](int u) {
+        UnitId id;
+        id.akey = u / (PO1 * PO2);
+        const int r = u - id.akey * (PO1 * PO2);
+        id.o1 = r / PO2;
+        id.o2 = r - id.o1 * PO2;
+        return id;
     };
-    auto unit_ptr = [&](int u) {
-        int akey, o1, o2;
-        decode(u, akey, o1, o2);
-        const int a = akey / NFR, fr = akey - a * NFR;
-        const int p4 = (FAM == FAM_D1) ? o2 : a, p5 = (FAM == FAM_D1) ? o1 : o2, p6 = (FAM == FAM_D1) ? a : o1;
+    auto advance = [&](UnitId id) {
+        if (++id.o2 == PO2) {
+            id.o2 = 0;
+            if (++id.o1 == PO1) {
+                id.o1 = 0;
+                ++id.akey;
+            }
+        }
+        return id;
+    };
+    auto unit_ptr = [&](const UnitId& id) {
+        const int a = id.akey / NFR, fr = id.akey - a * NFR;  // NFR is a compile-time constant
+        const int p4 = (FAM == FAM_D1) ? id.o2 : a, p5 = (FAM == FAM_D1) ? id.o1 : id.o2;
+        const int p6 = (FAM == FAM_D1) ? a : id.o1;
         return P.t3 + p4 * sp4 + p5 * sp5 + p6 * sp6 + fr * NF * sF + tbase;
     };
-    auto issue_B = [&](int u, double* dst) {  // B[k][y]
-        int akey, o1, o2;
-        decode(u, akey, o1, o2);
-        const double* src = (FAM == FAM_D1) ? opA + (int64_t)K * (o2 + (int64_t)P4 * o1)       // t2[k,p4,p5,h1]
-                                            : opB + (int64_t)K * H * (o1 + (int64_t)P6 * o2);  // v2[k,h3,p6,p5]
+    // B copies: element i = tid + m NT of [y][k] -> (y, k), first and step precomputed
+    const int by0 = tid / K, bk0 = tid - (tid / K) * K, bdy = NT / K, bdk = NT - (NT / K) * K;
+    auto issue_B = [&](const UnitId& id, double* dst) {  // B[k][y]
+        const double* src = (FAM == FAM_D1) ? opA + (int64_t)K * (id.o2 + (int64_t)P4 * id.o1)       // t2[k,p4,p5,h1]
+                                            : opB + (int64_t)K * H * (id.o1 + (int64_t)P6 * id.o2);  // v2[k,h3,p6,p5]
         const int stride_y = (FAM == FAM_D1) ? K * P4 * P5 : K;
+        int y = by0, k = bk0;
         for (int i = tid; i < H * K; i += NT) {
-            const int y = i / K, k = i - y * K;
             cp_async_8(dst + k * H + y, src + (int64_t)stride_y * y + k);
+            k += bdk;
+            if (k >= K) {
+                k -= K;
+                ++y;
+            }
+            y += bdy;
         }
     };
     auto load_tile = [&](const double* p, double (&x)[4][4]) {
@@ -2411,13 +2430,14 @@ __global__ void __launch_bounds__(SvGeo<H>::NT, SvGeo<H>::MINB) ccsdt_svs_kernel
     };
     if (lo >= hi) return;
     double x[4][4];  // [row][c]: xfast -> (y = row, x = c), else (x = row, y = c)
-    load_tile(unit_ptr(lo), x);
-    issue_B(lo, Bs);
+    UnitId cur = decode(lo);
+    load_tile(unit_ptr(cur), x);
+    issue_B(cur, Bs);
     cp_async_commit();
     int curA = -1;
     for (int u = lo; u < hi; ++u) {
-        int akey, o1, o2;
-        decode(u, akey, o1, o2);
+        const int akey = cur.akey;
+        const UnitId nxt = advance(cur);
         if (akey != curA) {  // stage A (sign folded) for (a, f range): once or twice per CTA
             __syncthreads();
             const int a = akey / NFR, f0 = (akey - a * NFR) * NF;
@@ -2451,15 +2471,15 @@ __global__ void __launch_bounds__(SvGeo<H>::NT, SvGeo<H>::MINB) ccsdt_svs_kernel
         cp_async_wait_all();
         __syncthreads();  // B(u) landed, A staged, the other B buffer is free
         const double* Bc = Bs + ((u - lo) & 1) * H * K;
-        if (u + 1 < hi) issue_B(u + 1, Bs + ((u + 1 - lo) & 1) * H * K);
+        if (u + 1 < hi) issue_B(nxt, Bs + ((u + 1 - lo) & 1) * H * K);
         cp_async_commit();
         double acc[4][4];
 #pragma unroll
         for (int r = 0; r < 4; ++r)
 #pragma unroll
             for (int c = 0; c < 4; ++c) acc[r][c] = x[r][c];
-        double* tp = unit_ptr(u);
-        if (u + 1 < hi) load_tile(unit_ptr(u + 1), x);
+        double* tp = unit_ptr(cur);
+        if (u + 1 < hi) load_tile(unit_ptr(nxt), x);
         const double* Ap = As + fl * RS + 4 * bx;
         const double* Bp = Bc + 4 * by;
 #pragma unroll 4
@@ -2483,6 +2503,7 @@ __global__ void __launch_bounds__(SvGeo<H>::NT, SvGeo<H>::MINB) ccsdt_svs_kernel
             st_cs2(tp + r * rstride, acc[r][0], acc[r][1]);
             st_cs2(tp + r * rstride + 2, acc[r][2], acc[r][3]);
         }
+        cur = nxt;
     }
 }
 
