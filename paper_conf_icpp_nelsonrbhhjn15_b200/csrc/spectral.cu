@@ -149,7 +149,7 @@ template <int P1, int NA, int AXIS, int R, int NT, typename T, typename Out, int
 __device__ __forceinline__ void apply_lines(const T* in, const T* opT, int nlines, Out out) {
     // fully unrolled chunks spill beyond P1 = 12 (ptxas, 255 registers at P1 = 13): those
     // keep the lane-strided loop
-    if constexpr (BC_WCHUNK && (UNR == 1 || P1 <= 12)) {
+    if constexpr (BC_WCHUNK && (UNR == 1 || P1 <= 12 || R <= 2)) {
         apply_lines_w<P1, NA, AXIS, R, NT, (bool)BC_SWP && UNR == 1, UNR>(in, opT, nlines, out);
         return;
     }
@@ -340,6 +340,12 @@ enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
 #define BC_SMALL_R 3  // sumfact3d lines per thread at P1 < 10 (measured: p=4 0.57 -> 0.65, p=5 0.56 -> 0.62,
                       // p=8 0.47 -> 0.53 of HBM vs R = 2; local_grad3 stays at R = 2)
 #endif
+#ifndef BC_R1011
+#define BC_R1011 4  // sumfact3d / local_grad3 lines per thread at P1 = 10, 11
+#endif
+#ifndef BC_SF2_R13
+#define BC_SF2_R13 3  // sumfact2d lines per thread at P1 >= 13
+#endif
 #ifndef BC_BIG_KB
 #define BC_BIG_KB 54
 #endif
@@ -360,7 +366,8 @@ struct SpecTable {
     static constexpr bool BIG = P1 >= 10;
     static constexpr bool SF3LG3 = KIND == K_SF3 || KIND == K_LG3;
     static constexpr bool MID = P1 == 12;  // sumfact3d / local_grad3: R = 3, 36 KiB (measured)
-    static constexpr int R = BIG ? (SF3LG3 ? (MID ? 3 : BC_BIG_R) : (KIND == K_SF2 ? 3 : 2))
+    static constexpr int R = BIG ? (SF3LG3 ? (MID ? 3 : (P1 <= 11 ? BC_R1011 : BC_BIG_R))
+                                           : (KIND == K_SF2 ? (P1 >= 13 ? BC_SF2_R13 : 3) : 2))
                                  : (KIND == K_SF3 ? BC_SMALL_R : 2);
     static constexpr int BUF_KB = BIG ? (SF3LG3 ? (MID ? 36 : BC_BIG_KB) : 18) : (KIND == K_LG3 ? 36 : 18);
     static constexpr bool PREFETCH = !(BIG && SF3LG3) || BC_BIG_PF;
