@@ -340,6 +340,9 @@ enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
 #define BC_SMALL_R 3  // sumfact3d lines per thread at P1 < 10 (measured: p=4 0.57 -> 0.65, p=5 0.56 -> 0.62,
                       // p=8 0.47 -> 0.53 of HBM vs R = 2; local_grad3 stays at R = 2)
 #endif
+#ifndef BC_LG3_DIRECT_UR
+#define BC_LG3_DIRECT_UR 0  // local_grad3: store ur from registers instead of in place + copy-out
+#endif
 #ifndef BC_R1011
 #define BC_R1011 4  // sumfact3d / local_grad3 lines per thread at P1 = 10, 11
 #endif
@@ -565,11 +568,19 @@ local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __rest
         apply_lines<P1, P1, 0, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
             st_cs(ut + gbase + Line<P1, P1, 0, T>::gofs(L, k), v);
         });
-        __syncthreads();
-        apply_lines<P1, P1, 2, R, NT>(in, opD, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
-        __syncthreads();
-        const int total = ne * G::NPTS;
-        for (int f = threadIdx.x; f < total; f += NT) st_cs(ur + gbase + f, in[smem_index<P1, P1, T>(f)]);
+        if constexpr (BC_LG3_DIRECT_UR) {
+            // ur rows stored straight from registers (lane-strided 8-byte stores; L2 merges the
+            // partial sectors of a warp's 13 consecutive stores)
+            apply_lines<P1, P1, 2, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
+                st_cs(ur + gbase + Line<P1, P1, 2, T>::gofs(L, k), v);
+            });
+        } else {
+            __syncthreads();
+            apply_lines<P1, P1, 2, R, NT>(in, opD, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
+            __syncthreads();
+            const int total = ne * G::NPTS;
+            for (int f = threadIdx.x; f < total; f += NT) st_cs(ur + gbase + f, in[smem_index<P1, P1, T>(f)]);
+        }
     });
 }
 
