@@ -343,6 +343,9 @@ enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
 #ifndef BC_LG3_DIRECT_UR
 #define BC_LG3_DIRECT_UR 0  // local_grad3: store ur from registers instead of in place + copy-out
 #endif
+#ifndef BC_E13_SF2
+#define BC_E13_SF2 0  // sumfact2d elements per group at P1 = 13 (0: derived, 12)
+#endif
 #ifndef BC_R1011
 #define BC_R1011 4  // sumfact3d / local_grad3 lines per thread at P1 = 10, 11
 #endif
@@ -376,7 +379,7 @@ struct SpecTable {
     static constexpr bool PREFETCH = !(BIG && SF3LG3) || BC_BIG_PF;
     // forced elements per group (0: derived from BUF_KB): P1 = 13: 3 x 169 = 507 lines on
     // 128 threads x R = 4 (1% idle lanes instead of 12% with E = 2 on 96 threads)
-    static constexpr int EF = (SF3LG3 && P1 == 13) ? BC_E13 : 0;
+    static constexpr int EF = (SF3LG3 && P1 == 13) ? BC_E13 : ((KIND == K_SF2 && P1 == 13) ? BC_E13_SF2 : 0);
     // unroll of the contracted-index loop: sumfact2d fully (its two stages fit the registers)
     static constexpr int UNROLL = (KIND == K_SF2 && BC_SF2_UNROLL && P1 >= 9) ? P1 : BC_NUNROLL;
 };

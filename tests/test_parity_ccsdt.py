@@ -35,10 +35,11 @@ def n3(ext):
 # includes shapes that take the 16-cube tensor-core (DMMA) path: hole extents 16/32/30 with
 # even k (ragged k chunk: 6, 10) and a ragged cube edge (30), and odd k (falls back to DFMA);
 # 16^3 / 24^3 holes with k <= 32 take the single-variant streaming kernel (ccsdt_svs_kernel):
-# unequal particle extents (A-name-major unit order), k = 7, 10, 16, 24, 32
+# unequal particle extents (A-name-major unit order), k = 1, 2, 7, 10, 16, 24, 32, one plane
 EXTS = [(3, 4, 5, 6, 2, 7, 3), (9, 17, 13, 5, 3, 4, 19), (8, 8, 8, 8, 8, 8, 8), (1, 1, 1, 1, 1, 1, 1),
         (16, 32, 16, 3, 4, 2, 6), (30, 16, 16, 2, 3, 2, 10), (16, 16, 30, 2, 2, 3, 10), (16, 16, 16, 2, 3, 2, 7),
-        (16, 16, 16, 3, 2, 4, 16), (16, 16, 16, 2, 4, 3, 32), (24, 24, 24, 2, 3, 2, 10), (24, 24, 24, 3, 1, 2, 24)]
+        (16, 16, 16, 3, 2, 4, 16), (16, 16, 16, 2, 4, 3, 32), (24, 24, 24, 2, 3, 2, 10), (24, 24, 24, 3, 1, 2, 24),
+        (16, 16, 16, 1, 1, 1, 1), (16, 16, 16, 1, 2, 1, 2)]
 
 
 @pytest.mark.parametrize("family", ["d1", "d2", "s1"])
