@@ -23,6 +23,16 @@
 // positions.  The cube has odd strides (1, BS+1, (BS+1)^2) on every axis, so the flush is
 // bank-conflict free for any permutation.  The (h1,h2,h3) <-> storage-position maps are
 // derived here from the generating rule of DESIGN.md R12 (not copied from the oracle).
+//
+// Kernels (dispatch in run_ccsdt / run_ccsdt_triples_energy):
+//   ccsdt_kernel<FAM,BS>        DFMA cube kernel, any shape (fallback)
+//   ccsdt_mma_kernel<FAM>       16-cube FP64 DMMA, cp.async staging (no tensor maps)
+//   ccsdt_tma_kernel<FAM>       16-cube DMMA, warp-specialised TMA ring (fused, tile 16)
+//   ccsdt_tma24_kernel<FAM>     exact 24-cube version (tile 24, fused and single variant)
+//   ccsdt_svs_kernel<FAM,H>     one d1/d2 variant, t3 streamed through registers (16^3 holes)
+//   ccsdt_sv16b_kernel<FAM>     the same with cp.async.bulk plane streaming (option)
+//   ccsdt_s1h_kernel<H> / ccsdt_s1_stream_kernel<RUN>   s1 streams (equal 16/24 holes / any)
+//   ccsdt_triples_energy_kernel / ccsdt_triples24_kernel  f4: 27 variants + energy (16- / 24-cube)
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
