@@ -2342,6 +2342,12 @@ __device__ __forceinline__ void st_cs2(double* p, double a, double b) {
     __stcs(reinterpret_cast<double2*>(p), make_double2(a, b));
 }
 
+#ifndef BC_SVS_MINB
+#define BC_SVS_MINB 2
+#endif
+#ifndef BC_SVS_PF
+#define BC_SVS_PF 1  // next unit's t3 tile prefetched into registers
+#endif
 // Geometry per hole extent H: a unit is (particle plane, range of NF values of f); thread
 // tiles are 4 x 4 over (x, y), so a unit has (H/4)^2 NF tiles = NT threads.
 template <int H>
@@ -2349,7 +2355,7 @@ struct SvGeo {
     static constexpr int NB = H / 4;               // tile blocks per hole axis
     static constexpr int NF = H == 16 ? 16 : 4;    // f values per unit
     static constexpr int NT = NB * NB * NF;        // 256 | 144
-    static constexpr int MINB = H == 16 ? 2 : 3;   // CTAs per SM (128 registers)
+    static constexpr int MINB = H == 16 ? BC_SVS_MINB : 3;  // CTAs per SM (128 registers at 2)
     static constexpr int NFR = H / NF;             // units per plane: 1 | 6
     static constexpr int RS = H + 2;               // A row stride (doubles, even)
     static constexpr int PS = NF * RS + 2;         // A k-plane stride
@@ -2483,13 +2489,14 @@ __global__ void __launch_bounds__(SvGeo<H>::NT, SvGeo<H>::MINB) ccsdt_svs_kernel
         const double* Bc = Bs + ((u - lo) & 1) * H * K;
         if (u + 1 < hi) issue_B(nxt, Bs + ((u + 1 - lo) & 1) * H * K);
         cp_async_commit();
+        if (!BC_SVS_PF && u != lo) load_tile(unit_ptr(cur), x);
         double acc[4][4];
 #pragma unroll
         for (int r = 0; r < 4; ++r)
 #pragma unroll
             for (int c = 0; c < 4; ++c) acc[r][c] = x[r][c];
         double* tp = unit_ptr(cur);
-        if (u + 1 < hi) load_tile(unit_ptr(nxt), x);
+        if (BC_SVS_PF && u + 1 < hi) load_tile(unit_ptr(nxt), x);
         const double* Ap = As + fl * RS + 4 * bx;
         const double* Bp = Bc + 4 * by;
 #pragma unroll 4
