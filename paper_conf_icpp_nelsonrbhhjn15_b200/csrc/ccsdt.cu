@@ -768,36 +768,6 @@ __device__ __forceinline__ void tma_flush_class(double* acc_s, double (&c)[4][2]
 
 // NSR: ring depth.  Single-variant launches (one stage per unit at tile 16) use NSR = 1
 // and 3 CTAs/SM: more units (t3 seeds) in flight for the HBM-bound case.
-// Unit index u = cube + ncubes * plane as six mixed-radix digits (cube coordinates along
-// the three hole positions, plane coordinates along the three particle positions), so a
-// persistent CTA advances u by gridDim.x with carries instead of six runtime divisions.
-struct UnitDigits {
-    int d[6];
-};
-__device__ __forceinline__ void unit_radix(const CcsdtParams& P, int (&r)[6]) {
-    r[0] = P.ncube[0]; r[1] = P.ncube[1]; r[2] = P.ncube[2];
-    r[3] = P.qe[3]; r[4] = P.qe[4]; r[5] = P.qe[5];
-}
-__device__ __forceinline__ UnitDigits unit_digits(int u, const int (&r)[6]) {  // divisions: once per CTA
-    UnitDigits x;
-#pragma unroll
-    for (int i = 0; i < 6; ++i) {
-        const int q = u / r[i];
-        x.d[i] = u - q * r[i];
-        u = q;
-    }
-    return x;
-}
-__device__ __forceinline__ void unit_add(UnitDigits& x, const UnitDigits& s, const int (&r)[6]) {
-    int carry = 0;
-#pragma unroll
-    for (int i = 0; i < 6; ++i) {
-        int v = x.d[i] + s.d[i] + carry;
-        carry = v >= r[i];
-        x.d[i] = carry ? v - r[i] : v;
-    }
-}
-
 template <int FAM, int NSR = TmaGeo::NS, int MINB = 2>
 __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __grid_constant__ CcsdtParams P,
                                                                      const __grid_constant__ TmaMaps M, int units) {
@@ -827,27 +797,23 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
     const int nchunk = (K + KC - 1) / KC;
     const int nstage = P.nentry * nchunk;
 
-    int rad[6];
-    unit_radix(P, rad);
-    const UnitDigits ustep = unit_digits(gridDim.x, rad);
-    auto decode_d = [&](const UnitDigits& x, int* o, int* len, int* qv) {
-#pragma unroll
-        for (int q = 0; q < 3; ++q) {
-            o[q] = x.d[q] * BS;
-            len[q] = min(BS, P.qe[q] - o[q]);
-            qv[q] = x.d[3 + q];
-        }
+    auto decode = [&](int u, int* o, int* len, int* qv) {
+        const int cube = u % ncubes, plane = u / ncubes;
+        o[0] = (cube % P.ncube[0]) * BS;
+        o[1] = ((cube / P.ncube[0]) % P.ncube[1]) * BS;
+        o[2] = (cube / (P.ncube[0] * P.ncube[1])) * BS;
+        for (int q = 0; q < 3; ++q) len[q] = min(BS, P.qe[q] - o[q]);
+        qv[0] = plane % P.qe[3];
+        qv[1] = (plane / P.qe[3]) % P.qe[4];
+        qv[2] = plane / (P.qe[3] * P.qe[4]);
     };
-    (void)ncubes;
 
     if (warp == TG::NCW) {
         // ================================ producer: lane 0 arms the stage, lanes issue copies
         int g = 0;
-        UnitDigits ud = unit_digits(blockIdx.x, rad);
-        for (int u = blockIdx.x; u < units; u += gridDim.x, unit_add(ud, ustep, rad)) {
+        for (int u = blockIdx.x; u < units; u += gridDim.x) {
             int o[3], len[3], qv[3];
-            decode_d(ud, o, len, qv);
-            int e = 0, kc_i = 0;
+            decode(u, o, len, qv);
             for (int st = 0; st < nstage; ++st, ++g) {
                 const int slot = g % NS;
                 const uint32_t full = bar_full + 8 * slot;
@@ -856,17 +822,13 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
                     mbar_expect_tx(full, TG::STAGE_BYTES);
                 }
                 __syncwarp();
-                const int k0 = kc_i * KC;
-                if (++kc_i == nchunk) kc_i = 0;
-                const int e_cur = e;
-                if (kc_i == 0) ++e;
-                const int c = P.ecls[e_cur];
-                auto opos = [&](int pos) { return pos == 0 ? o[0] : (pos == 1 ? o[1] : o[2]); };
-                const int O1 = opos(P.hpos[c][0]), O2 = opos(P.hpos[c][1]), O3 = opos(P.hpos[c][2]);
+                const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
+                const int c = P.ecls[e];
+                const int O1 = o[P.hpos[c][0]], O2 = o[P.hpos[c][1]], O3 = o[P.hpos[c][2]];
                 auto pick = [&](int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
-                const int p4 = pick(P.ppos[e_cur][0]), p5 = pick(P.ppos[e_cur][1]), p6 = pick(P.ppos[e_cur][2]);
+                const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
                 const uint32_t A = st_u32 + slot * TG::STAGE_BYTES;
-                tma_issue_stage<FAM>(&M.a[e_cur], &M.b[e_cur], A, A + TG::A_BYTES, full, lane, O1, O2, O3, p4, p5, p6, k0);
+                tma_issue_stage<FAM>(&M.a[e], &M.b[e], A, A + TG::A_BYTES, full, lane, O1, O2, O3, p4, p5, p6, k0);
             }
         }
         return;
@@ -897,15 +859,9 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
     };
     const bool full_cubes = P.qe[0] % BS == 0 && P.qe[1] % BS == 0 && P.qe[2] % BS == 0;
     int g = 0;
-    UnitDigits ud = unit_digits(blockIdx.x, rad);
     for (int u = blockIdx.x; u < units; u += gridDim.x) {
         int o[3], len[3], qv[3];
-        decode_d(ud, o, len, qv);
-        UnitDigits udn = ud;
-        unit_add(udn, ustep, rad);
-        const UnitDigits ud_this = ud;
-        ud = udn;  // the next iteration's unit
-        (void)ud_this;
+        decode(u, o, len, qv);
         const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
                               (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
         const int nvol = len[0] * len[1] * len[2];
@@ -980,7 +936,7 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
             const int un = u + gridDim.x;
             if (un < units) {
                 int on[3], lenn[3], qvn[3];
-                decode_d(udn, on, lenn, qvn);
+                decode(un, on, lenn, qvn);
                 const int64_t pbn = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
                                     (qvn[0] + (int64_t)P.qe[3] * (qvn[1] + (int64_t)P.qe[4] * qvn[2]));
                 const double* srcg = P.t3 + pbn + (on[0] + q0) + (int64_t)Q0 * ((on[1] + q1) + (int64_t)P.qe[1] * on[2]);

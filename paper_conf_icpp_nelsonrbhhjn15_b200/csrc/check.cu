@@ -71,7 +71,23 @@ __global__ void __launch_bounds__(RED_NT) energy_partial(EnergyDims d, const dou
         const int p6 = pl % d.p6, p5 = (pl / d.p6) % d.p5, p4 = pl / (d.p6 * d.p5);
         const double a6 = f6[p6], a5 = f5[p5], a4 = f4[p4];
         const double* row = t3 + (int64_t)pl * nh;
-        for (int i = threadIdx.x; i < nh; i += RED_NT) {
+        int i = threadIdx.x;
+        if (tab) {
+            // EN_UNR independent loads in flight per thread before the dependent divisions:
+            // one load per iteration left the pass latency-bound (≈0.3 of HBM at tile 16).
+            constexpr int EN_UNR = 8;
+            for (; i + (EN_UNR - 1) * RED_NT < nh; i += EN_UNR * RED_NT) {
+                double t[EN_UNR];
+#pragma unroll
+                for (int u = 0; u < EN_UNR; ++u) t[u] = __ldcs(row + i + u * RED_NT);
+#pragma unroll
+                for (int u = 0; u < EN_UNR; ++u) {
+                    const double den = ((dh[i + u * RED_NT] - a6) - a5) - a4;
+                    s += t[u] * t[u] / den;
+                }
+            }
+        }
+        for (; i < nh; i += RED_NT) {
             double h;
             if (tab) {
                 h = dh[i];

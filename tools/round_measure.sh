@@ -13,4 +13,8 @@ for k in ${KERNELS:-local_grad3_kernel sumfact3d_kernel sumfact2d_kernel ccsdt_t
   ncu --set full --clock-control none --import-source on -k regex:$k -s 2 -c 1 -o $OUT/prof_$k -f \
       python bench.py --no-cpu --no-e2e --steps 1 --warmup 3 > /dev/null 2> $OUT/prof_$k.err
 done
+for r in $OUT/*.ncu-rep; do
+  [ -e "$r" ] || continue
+  ncu -i "$r" --page raw --csv > "${r%.ncu-rep}.raw.csv" 2>/dev/null && rm -f "$r"
+done
 ls -la $OUT

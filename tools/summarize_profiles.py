@@ -53,9 +53,15 @@ WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
 traffic = {}
 lines += ["", "## ncu --set full (one launch each)", ""]
 for f in sorted(os.listdir(G)):
-    if not f.endswith(".ncu-rep"):
+    # .ncu-rep (read here) or its --page raw --csv export (written on the box by
+    # tools/round_measure.sh so gpurun_out/ stays under the copy-back limit)
+    if f.endswith(".ncu-rep"):
+        raw = subprocess.run(["ncu", "-i", os.path.join(G, f), "--page", "raw", "--csv"],
+                             capture_output=True, text=True).stdout
+    elif f.endswith(".raw.csv"):
+        raw = open(os.path.join(G, f)).read()
+    else:
         continue
-    raw = subprocess.run(["ncu", "-i", os.path.join(G, f), "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rr = list(csv.reader(io.StringIO(raw)))
     if len(rr) < 3:
         continue
