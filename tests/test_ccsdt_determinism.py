@@ -5,8 +5,9 @@ order: per class, one owning thread adds its DMMA accumulator, and the classes r
 entry order. Without a race, repeated launches on identical inputs are therefore bitwise
 identical. A flush or seed race shows up as a few hundred t3 elements that differ between
 runs (the reverted division-free decode). The small parity tests never
-reached that state; this test repeats the bench's configuration (tile 16, 8 blocks, all 9
-variants of d1 then d2) and compares t3 across runs without calling the oracle.
+reached that state. This test repeats the bench's configuration (tile 16, 8 blocks, all 9
+variants of d1 then d2), plus the exact-24-cube kernel (tile 24, 2 blocks), and compares
+t3 across runs without calling the oracle.
 """
 import pytest
 import torch
@@ -18,7 +19,7 @@ pytestmark = pytest.mark.gpu
 REPEATS = 6
 
 
-@pytest.mark.parametrize("tile,blocks", [(16, 8)])
+@pytest.mark.parametrize("tile,blocks", [(16, 8), (24, 2)])
 def test_fused_repeat_bitwise(tile, blocks):
     dev = torch.device("cuda:0")
     f64 = torch.float64
