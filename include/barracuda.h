@@ -186,6 +186,18 @@ int bc_fill(int kind, uint64_t seed, uint64_t tensor_id, uint64_t offset, int64_
 int bc_fill_f32(int kind, uint64_t seed, uint64_t tensor_id, uint64_t offset, int64_t n,
                 double lo, double hi, float* out, void* stream);
 
+/* ===================================================================== measurement */
+
+/* FP64 peak probe (a measurement utility, not a method operation): launches a kernel of
+ * independent FP64 chains so the bench can time the FP64 roofline denominators live
+ * (DESIGN.md §4): kind 0 = DFMA (fma.rn.f64), kind 1 = DMMA (mma.sync.m8n8k4.f64).
+ * iters in [1, 2^20] scales the work; *flops (HOST pointer) receives the number of
+ * floating-point operations the launch performs (the caller times it with CUDA events).
+ * scratch: device, >= bc_probe_scratch_doubles() doubles (receives the chain results). */
+int bc_probe_fp64(int kind, int iters, double* scratch, int64_t scratch_doubles, double* flops,
+                  void* stream);
+int64_t bc_probe_scratch_doubles(void);
+
 /* ===================================================================== misc */
 
 const char* bc_status_string(int status);

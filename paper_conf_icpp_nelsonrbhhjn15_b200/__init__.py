@@ -22,7 +22,7 @@ from ._abi import BC_CHECK_WS_DOUBLES, TileDims, lib
 __all__ = [
     "BarracudaError", "sumfact3d", "sumfact2d", "local_grad3", "local_grad3_t", "ax_e",
     "ccsdt", "ccsdt_fused", "ccsdt_triples_energy", "check_sumsq", "check_energy", "fill", "launch_count",
-    "reset_launch_count", "LIB_PATH",
+    "reset_launch_count", "probe_fp64_tflops", "LIB_PATH",
 ]
 
 LIB_PATH = _abi.LIB_PATH
@@ -232,6 +232,29 @@ def fill(out: torch.Tensor, tensor_id: int, kind: int = KIND_REAL, seed: int = 2
     _check(fn(int(kind), int(seed), int(tensor_id), int(offset), out.numel(), float(lo), float(hi),
               _dev(out, out.dtype, "out"), _stream(out)), "bc_fill")
     return out
+
+
+def probe_fp64_tflops(kind: str, device=None, iters: int = 2000, reps: int = 3) -> float:
+    """Measured FP64 throughput (TFLOP/s) of the DFMA ("dfma") or DMMA ("dmma") pipe on
+    `device`: best of `reps` timed launches of bc_probe_fp64 (CUDA events)."""
+    dev = torch.device("cuda") if device is None else torch.device(device)
+    k = {"dfma": 0, "dmma": 1}[kind]
+    n = int(lib.bc_probe_scratch_doubles())
+    scratch = torch.empty(n, dtype=torch.float64, device=dev)
+    flops = ctypes.c_double(0.0)
+    st = torch.cuda.current_stream(dev)
+    sp = ctypes.c_void_p(st.cuda_stream)
+    _check(lib.bc_probe_fp64(k, 10, _dev(scratch, torch.float64, "scratch"), n, ctypes.byref(flops), sp),
+           "bc_probe_fp64")
+    best = 0.0
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(st)
+        _check(lib.bc_probe_fp64(k, iters, scratch.data_ptr(), n, ctypes.byref(flops), sp), "bc_probe_fp64")
+        e1.record(st)
+        e1.synchronize()
+        best = max(best, flops.value / (e0.elapsed_time(e1) * 1e-3) / 1e12)
+    return best
 
 
 def launch_count() -> int:

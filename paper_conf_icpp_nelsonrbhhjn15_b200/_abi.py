@@ -49,6 +49,8 @@ _SIGS = {
     "bc_check_energy": [ctypes.POINTER(TileDims), _vp, _vp, _vp, _vp, _vp],
     "bc_fill": [_i32, _u64, _u64, _u64, _i64, _d, _d, _vp, _vp],
     "bc_fill_f32": [_i32, _u64, _u64, _u64, _i64, _d, _d, _vp, _vp],
+    "bc_probe_fp64": [_i32, _i32, _vp, _i64, ctypes.POINTER(_d), _vp],
+    "bc_probe_scratch_doubles": [],
     "bc_status_string": [_i32],
     "bc_last_cuda_error": [],
     "bc_version": [],
@@ -64,6 +66,7 @@ for _name, _args in _SIGS.items():
     _f.restype = _i32
 lib.bc_status_string.restype = ctypes.c_char_p
 lib.bc_launch_count.restype = _i64
+lib.bc_probe_scratch_doubles.restype = _i64
 lib.bc_reset_launch_count.restype = None
 
 BC_CHECK_WS_DOUBLES = 1024

@@ -25,8 +25,9 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
                              const double* const* t2d1, const double* const* v2d1, const double* const* t2d2,
                              const double* const* v2d2, const double* eps_h, const double* eps_p, double* ws,
                              cudaStream_t s);
-void set_triples_dump(double* p);
 int run_sumsq(int64_t n, const double* x, double* ws, cudaStream_t s);
+int run_probe_fp64(int kind, int iters, double* scratch, double* flops, cudaStream_t s);
+int probe_scratch_doubles();
 int run_energy(const int* ext7, const double* t3, const double* eh, const double* ep, double* ws, cudaStream_t s);
 template <typename T>
 int run_fill(int kind, uint64_t seed, uint64_t tid, uint64_t offset, int64_t n, double lo, double hi, T* out,
@@ -313,9 +314,6 @@ int bc_ccsdt_triples_energy(const bc_tile_dims* d, const double* const t1[9], co
     return run_ccsdt_triples_energy(e, t1, v2s1, t2d1, v2d1, t2d2, v2d2, eps_h, eps_p, ws, as_stream(stream));
 }
 
-/* debug hook (not in barracuda.h): make bc_ccsdt_triples_energy also store its t3 */
-void bc_debug_triples_dump(double* t3) { set_triples_dump(t3); }
-
 int bc_check_sumsq(int64_t n, const double* x, double* ws, void* stream) {
     BC_REQUIRE(n >= 0 && ws, BC_ERR_ARG);
     BC_REQUIRE(n == 0 || x, BC_ERR_ARG);
@@ -352,6 +350,14 @@ int bc_fill_f32(int kind, uint64_t seed, uint64_t tensor_id, uint64_t offset, in
     BC_REQUIRE(aligned(out, 4), BC_ERR_ALIGN);
     return run_fill<float>(kind, seed, tensor_id, offset, n, lo, hi, out, as_stream(stream));
 }
+
+int bc_probe_fp64(int kind, int iters, double* scratch, int64_t scratch_doubles, double* flops, void* stream) {
+    BC_REQUIRE((kind == 0 || kind == 1) && iters >= 1 && iters <= (1 << 20) && scratch && flops, BC_ERR_ARG);
+    BC_REQUIRE(scratch_doubles >= probe_scratch_doubles(), BC_ERR_ARG);
+    BC_REQUIRE(aligned(scratch, 8), BC_ERR_ALIGN);
+    return run_probe_fp64(kind, iters, scratch, flops, as_stream(stream));
+}
+int64_t bc_probe_scratch_doubles(void) { return probe_scratch_doubles(); }
 
 const char* bc_status_string(int status) {
     switch (status) {

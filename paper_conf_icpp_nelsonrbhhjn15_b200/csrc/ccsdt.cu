@@ -623,6 +623,20 @@ __device__ __forceinline__ void named_bar_sync(int id, int n) {
     asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(n) : "memory");
 }
 
+// Consumer warp releases a ring slot it has finished reading.  The slot's next contents
+// are written by TMA, i.e. by the ASYNC proxy, while the consumers read it with ordinary
+// ld.shared (the GENERIC proxy); the mbarrier release/acquire pair orders the two only
+// after a proxy fence: without `fence.proxy.async`, ptxas issues the arrive while the
+// stage's last ld.shared are still in flight and the producer's refill can overwrite a
+// fragment before it is read (measured: 183 of 200 repeat runs of the tile-16 fused
+// kernel corrupted 128-1648 t3 values, one warp m-tile each; with the fence 0 of 200 —
+// DESIGN.md §4.2).  Every lane fences its own reads, then lane 0 arrives for the warp.
+__device__ __forceinline__ void release_slot(uint32_t bar_empty_slot, int lane) {
+    asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+    __syncwarp();
+    if (lane == 0) mbar_arrive(bar_empty_slot);
+}
+
 // fragment loads as volatile asm: kept in program order relative to the (volatile) DMMAs,
 // so a stage's fragments are all loaded into distinct registers before its first DMMA
 // (plain loads let ptxas reuse one register per fragment and expose the LDS latency
@@ -686,7 +700,7 @@ __device__ __forceinline__ void tma_issue_stage(const CUtensorMap* ma, const CUt
 // tensor extent arrives zero-filled by TMA)
 template <int FE>
 __device__ __forceinline__ void tma_consume_stage(const unsigned char* A, const unsigned char* B, uint32_t smask,
-                                                  double (&c)[4][2][2], int warp, int gq, int tq) {
+                                                      double (&c)[4][2][2], int warp, int gq, int tq) {
     double bfa[TmaGeo::KC / 4][2], afa[TmaGeo::KC / 4][4];
     // an 8-row step of a 64B-swizzled operand is +512 B with the same XOR pattern, so the
     // n-/m-tiles are immediate offsets from one base per k-step
@@ -768,6 +782,31 @@ __device__ __forceinline__ void tma_flush_class(double* acc_s, double (&c)[4][2]
 
 // NSR: ring depth.  Single-variant launches (one stage per unit at tile 16) use NSR = 1
 // and 3 CTAs/SM: more units (t3 seeds) in flight for the HBM-bound case.
+// Unit index u = cube + ncubes * plane as six mixed-radix digits (cube coordinates along
+// the three hole positions, plane coordinates along the three particle positions), so a
+// persistent CTA advances u by gridDim.x with carries instead of six runtime divisions.
+struct UnitDigits {
+    int d[6];
+};
+__device__ __forceinline__ UnitDigits unit_digits(int u, const int (&r)[6]) {  // divisions: once per CTA
+    UnitDigits x;
+#pragma unroll
+    for (int i = 0; i < 6; ++i) {
+        const int q = u / r[i];
+        x.d[i] = u - q * r[i];
+        u = q;
+    }
+    return x;
+}
+__device__ __forceinline__ void unit_add(UnitDigits& x, const UnitDigits& s, const int (&r)[6]) {
+    int carry = 0;
+#pragma unroll
+    for (int i = 0; i < 6; ++i) {
+        const int v = x.d[i] + s.d[i] + carry;
+        carry = v >= r[i];
+        x.d[i] = carry ? v - r[i] : v;
+    }
+}
 template <int FAM, int NSR = TmaGeo::NS, int MINB = 2>
 __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __grid_constant__ CcsdtParams P,
                                                                      const __grid_constant__ TmaMaps M, int units) {
@@ -792,28 +831,29 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
     }
     __syncthreads();
 
-    const int ncubes = P.ncube[0] * P.ncube[1] * P.ncube[2];
     const int K = P.ext[N_K];
     const int nchunk = (K + KC - 1) / KC;
     const int nstage = P.nentry * nchunk;
 
-    auto decode = [&](int u, int* o, int* len, int* qv) {
-        const int cube = u % ncubes, plane = u / ncubes;
-        o[0] = (cube % P.ncube[0]) * BS;
-        o[1] = ((cube / P.ncube[0]) % P.ncube[1]) * BS;
-        o[2] = (cube / (P.ncube[0] * P.ncube[1])) * BS;
-        for (int q = 0; q < 3; ++q) len[q] = min(BS, P.qe[q] - o[q]);
-        qv[0] = plane % P.qe[3];
-        qv[1] = (plane / P.qe[3]) % P.qe[4];
-        qv[2] = plane / (P.qe[3] * P.qe[4]);
+    int rad[6] = {P.ncube[0], P.ncube[1], P.ncube[2], P.qe[3], P.qe[4], P.qe[5]};
+    const UnitDigits ustep = unit_digits(gridDim.x, rad);
+    auto decode_d = [&](const UnitDigits& x, int* o, int* len, int* qv) {
+#pragma unroll
+        for (int q = 0; q < 3; ++q) {
+            o[q] = x.d[q] * BS;
+            len[q] = min(BS, P.qe[q] - o[q]);
+            qv[q] = x.d[3 + q];
+        }
     };
 
     if (warp == TG::NCW) {
         // ================================ producer: lane 0 arms the stage, lanes issue copies
         int g = 0;
-        for (int u = blockIdx.x; u < units; u += gridDim.x) {
+        UnitDigits ud = unit_digits(blockIdx.x, rad);
+        for (int u = blockIdx.x; u < units; u += gridDim.x, unit_add(ud, ustep, rad)) {
             int o[3], len[3], qv[3];
-            decode(u, o, len, qv);
+            decode_d(ud, o, len, qv);
+            int e = 0, kc_i = 0;
             for (int st = 0; st < nstage; ++st, ++g) {
                 const int slot = g % NS;
                 const uint32_t full = bar_full + 8 * slot;
@@ -822,13 +862,18 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
                     mbar_expect_tx(full, TG::STAGE_BYTES);
                 }
                 __syncwarp();
-                const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
-                const int c = P.ecls[e];
-                const int O1 = o[P.hpos[c][0]], O2 = o[P.hpos[c][1]], O3 = o[P.hpos[c][2]];
+                const int k0 = kc_i * KC;
+                if (++kc_i == nchunk) kc_i = 0;
+                const int e_cur = e;
+                if (kc_i == 0) ++e;
+                const int c = P.ecls[e_cur];
+                auto opos = [&](int pos) { return pos == 0 ? o[0] : (pos == 1 ? o[1] : o[2]); };
+                const int O1 = opos(P.hpos[c][0]), O2 = opos(P.hpos[c][1]), O3 = opos(P.hpos[c][2]);
                 auto pick = [&](int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
-                const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
+                const int p4 = pick(P.ppos[e_cur][0]), p5 = pick(P.ppos[e_cur][1]), p6 = pick(P.ppos[e_cur][2]);
                 const uint32_t A = st_u32 + slot * TG::STAGE_BYTES;
-                tma_issue_stage<FAM>(&M.a[e], &M.b[e], A, A + TG::A_BYTES, full, lane, O1, O2, O3, p4, p5, p6, k0);
+                tma_issue_stage<FAM>(&M.a[e_cur], &M.b[e_cur], A, A + TG::A_BYTES, full, lane, O1, O2, O3, p4, p5, p6,
+                                     k0);
             }
         }
         return;
@@ -859,9 +904,11 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
     };
     const bool full_cubes = P.qe[0] % BS == 0 && P.qe[1] % BS == 0 && P.qe[2] % BS == 0;
     int g = 0;
+    UnitDigits ud = unit_digits(blockIdx.x, rad);
     for (int u = blockIdx.x; u < units; u += gridDim.x) {
         int o[3], len[3], qv[3];
-        decode(u, o, len, qv);
+        decode_d(ud, o, len, qv);
+        unit_add(ud, ustep, rad);  // ud: the CTA's next unit (u + gridDim.x)
         const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
                               (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
         const int nvol = len[0] * len[1] * len[2];
@@ -896,8 +943,7 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
             const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
             const unsigned char* B = A + TG::A_BYTES;
             tma_consume_stage<FAM>(A, B, smask, c, warp, gq, tq);
-            __syncwarp();
-            if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
+            release_slot(bar_empty + 8 * slot, lane);
             const bool last_chunk = (++kc_i == nchunk);
             const int e_cur = e;
             if (last_chunk) {
@@ -936,7 +982,7 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
             const int un = u + gridDim.x;
             if (un < units) {
                 int on[3], lenn[3], qvn[3];
-                decode(un, on, lenn, qvn);
+                decode_d(ud, on, lenn, qvn);
                 const int64_t pbn = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
                                     (qvn[0] + (int64_t)P.qe[3] * (qvn[1] + (int64_t)P.qe[4] * qvn[2]));
                 const double* srcg = P.t3 + pbn + (on[0] + q0) + (int64_t)Q0 * ((on[1] + q1) + (int64_t)P.qe[1] * on[2]);
@@ -1237,8 +1283,7 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
                 for (int mi = 0; mi < 9; ++mi)
 #pragma unroll
                     for (int ni = 0; ni < 3; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[ks][mi], bf[ks][ni]);
-            __syncwarp();
-            if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
+            release_slot(bar_empty + 8 * slot, lane);
             const bool last_chunk = (++kc_i == nchunk);
             const int e_cur = e;
             if (last_chunk) {
@@ -1382,7 +1427,6 @@ struct TripParams {
     const double* eps_h;
     const double* eps_p;
     double* ws;
-    double* dump;  // debug only (bc_debug_triples_dump): store the t3 cube, canonical layout
 };
 struct TripMaps {
     CUtensorMap a[TRIP_MAXE];
@@ -1509,8 +1553,7 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const 
             const bool d1 = P.efam[e] == FAM_D1;
             if (d1) tma_consume_stage<FAM_D1>(A, B, P.smask[e], c, warp, gq, tq);
             else tma_consume_stage<FAM_D2>(A, B, P.smask[e], c, warp, gq, tq);
-            __syncwarp();
-            if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
+            release_slot(bar_empty + 8 * slot, lane);
             if (k0 + KC >= K && (e + 1 == P.nentry || P.ecls[e + 1] != P.ecls[e])) {
                 named_bar_sync(1, 256);  // no two classes flush concurrently (see ccsdt_tma_kernel)
                 if (d1) tma_flush_class<FAM_D1>(acc_s, c, P.hpos[P.ecls[e]], warp, gq, tq);
@@ -1552,9 +1595,6 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const 
             const double den = ((((eh3[o[0] + q0] + eh2[o[1] + q1]) + eh1[o[2] + q2]) - ep6[qv[0]]) - ep5[qv[1]]) -
                                ep4[qv[2]];
             energy += t * t / den;
-            if (P.dump)
-                P.dump[(o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * ((o[2] + q2) +
-                       (int64_t)P.qe[2] * (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]))))] = t;
         }
     }
     // consumer-only block reduction (the producer warp has left)
@@ -1739,8 +1779,7 @@ __global__ void __launch_bounds__(Trip24Geo::NT, 1) ccsdt_triples24_kernel(const
             const bool d1 = P.efam[e] == FAM_D1;
             if (d1) t24_consume<FAM_D1>(A, B, P.smask[e], c, warp, gq, tq);
             else t24_consume<FAM_D2>(A, B, P.smask[e], c, warp, gq, tq);
-            __syncwarp();
-            if (lane == 0) mbar_arrive(bar_empty + 8 * slot);
+            release_slot(bar_empty + 8 * slot, lane);
             const bool last_chunk = (++kc_i == nchunk);
             const int e_cur = e;
             if (last_chunk) {
@@ -1796,9 +1835,6 @@ __global__ void __launch_bounds__(Trip24Geo::NT, 1) ccsdt_triples24_kernel(const
                 const double t = xp[C2 * q2];
                 const double den = (((h32 + eh1[q2]) - e6) - e5) - e4;
                 energy += t * t / den;
-                if (P.dump)
-                    P.dump[q0 + (int64_t)BS * (q1 + (int64_t)BS * (q2 + (int64_t)BS * (qv[0] + (int64_t)P.qe[3] *
-                           (qv[1] + (int64_t)P.qe[4] * qv[2]))))] = t;
             }
         }
     }
@@ -1812,8 +1848,6 @@ __global__ void __launch_bounds__(Trip24Geo::NT, 1) ccsdt_triples24_kernel(const
     }
 }
 
-static double* g_triples_dump = nullptr;  // debug only
-void set_triples_dump(double* p) { g_triples_dump = p; }
 
 // Host: d1/d2 entries grouped by class (d1 classes 0-2, d2 classes 3-5), s1 list.
 int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const double* const* v2s1,
@@ -1834,7 +1868,6 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
     P.eps_h = eps_h;
     P.eps_p = eps_p;
     P.ws = ws;
-    P.dump = g_triples_dump;
     int n = 0, ncls = 0;
     const double* const* tA[2] = {t2d1, t2d2};
     const double* const* vB[2] = {v2d1, v2d2};
