@@ -2,15 +2,22 @@
 """Benchmark: fp64 GFLOP/s of one pass of the whole hot path.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl barracuda|reference]
+                    [--scaling weak|strong]
 
-N > 1 is launched by the driver with torchrun (one process per GPU, NCCL).  Each rank owns
-its own slice of the global batch (weak scaling; no data-path collective — only the
-check-scalar SUM and the max-over-ranks of the timing cross GPUs).  Rank 0 prints ONE JSON
-line.  The default workload is BASELINE.json configs[1] (Nekbone local_grad3, p=12,
-N=262,144 elements per GPU) with every other §8(a) row run over the same batch in the same
-step (sumfact3d, sumfact2d, CCSD(T) d1/d2 fused tile 16, check scalars).
+N > 1 is launched by the driver with torchrun (one process per GPU, NCCL).  Units are
+independent: with --scaling weak (default) each rank owns its own
+slice of the global batch; with --scaling strong the global batch (--n-elem elements,
+--blocks CCSD(T) blocks) is split over the ranks by dist.shard().  No data-path
+collective: only the check-scalar SUM, the flop SUM and the max-over-ranks of the timing
+cross GPUs.  Rank 0 prints ONE JSON line.  The default workload is BASELINE.json
+configs[1] (Nekbone local_grad3, p=12, N=262,144 elements) with every other §8(a) row run
+over the same batch in the same step (sumfact3d, sumfact2d, CCSD(T) d1/d2 fused tile 16,
+check scalars), plus per-config rows (BASELINE configs 1, 3, 4, 5) measured in the same
+run after the timed step.
 
-Only the cpu_baseline leg and --impl reference execute the oracle (oracle/), on host cores.
+The oracle (oracle/) is executed only by the cpu_baseline leg and by --impl reference;
+those legs import only `oracle`, `synthetic` and `accounting` (never the product
+package, so libbarracuda.so is not loaded there).
 """
 from __future__ import annotations
 
@@ -28,9 +35,10 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
-FP64_PEAK_TFLOPS = 37.2  # 148 SMs x 64 FP64 FMA/clk x 2 x 1.965 GHz; measured 37.1 (DMMA) / 34.2 (DFMA),
-#                          tools/fp64_peak.cu -> profiles/fp64_peak_r01.txt
-METRIC = "fp64 GFLOP/s & % of HBM/FP64 roofline for batched small contractions, 1-8 GPU"
+import accounting as acct  # noqa: E402
+from accounting import METRIC, StepConfig  # noqa: E402
+
+FP64_NOMINAL_TFLOPS = 37.2  # 148 SMs x 64 FP64 FMA/clk x 2 x 1.965 GHz (only if the live probe fails)
 
 
 def load_peaks():
@@ -48,6 +56,17 @@ def load_traffic():
         with open(p) as f:
             return json.load(f)
     return {}
+
+
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 class ClockSampler:
@@ -101,24 +120,30 @@ class ClockSampler:
                     reasons.add(nm)
         if not sm:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
-        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": max(mx), "reasons": sorted(reasons), "samples": len(sm)}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "samples": len(sm), "gpu": self.index}
+
+
+def env_rank():
+    return int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1"))
 
 
 # ---------------------------------------------------------------------------- oracle legs
-def oracle_sample_rate(cfg, n_spec: int = 8192, ccsdt_blocks: int = 1):
-    """Time the oracle (as it stands) on a bounded sample of the step and return the
+def oracle_sample(cfg: StepConfig, n_spec: int = 8192, ccsdt_blocks: int = 1, threads: int | None = None):
+    """Time the oracle (as it stands) on a bounded sample of the step: n_spec elements of
+    each spectral kernel and `ccsdt_blocks` CCSD(T) blocks of d1+d2 fused.  Returns the
     step-equivalent GFLOP/s (each kernel's sample rate weighted by its share of the full
-    step's flops), the sample description and the seconds spent."""
+    step's flops), the sample description, the seconds spent and per-kernel GFLOP/s.
+    Imports only oracle / synthetic / accounting."""
     import oracle
     import synthetic as syn
-    from paper_conf_icpp_nelsonrbhhjn15_b200.workload import flops_bytes
 
-    P1 = cfg.P1
-    fb = flops_bytes(cfg)
+    if threads is not None:
+        oracle.set_threads(threads)
+    P1, t = cfg.P1, cfg.tile
     U = syn.elements(syn.TID["U"], P1, np.arange(n_spec))
     A, B, C = (syn.tensor(syn.TID[n], (P1, P1)) for n in ("A", "B", "C"))
     D = syn.gll_derivative(cfg.p)
-    t = cfg.tile
     ext = (t,) * 7
     t3 = syn.tensor(syn.ccsdt_block_tid(syn.TID["T3"], 0, 0), (t ** 6,))
     ops = {fam: ([syn.tensor(syn.ccsdt_block_tid(syn.TID["T2"] + (0 if fam == "d1" else 200000), v, 0), (t ** 4,))
@@ -135,11 +160,10 @@ def oracle_sample_rate(cfg, n_spec: int = 8192, ccsdt_blocks: int = 1):
         for _ in range(ccsdt_blocks):
             oracle.ccsdt_fused(fam, ext, t3, *ops[fam])
         secs[f"ccsdt_{fam}_fused"] = time.perf_counter() - t0
-    sample_flops = {"local_grad3": fb["local_grad3"][0] * n_spec / cfg.n_elem,
-                    "sumfact3d": fb["sumfact3d"][0] * n_spec / cfg.n_elem,
-                    "sumfact2d": fb["sumfact2d"][0] * n_spec / cfg.n_elem,
-                    **{f"ccsdt_{f}_fused": fb[f"ccsdt_{f}_fused"][0] * ccsdt_blocks for f in cfg.families}}
-    full_flops = {k: fb[k][0] * (cfg.blocks if k.startswith("ccsdt") else 1) for k in sample_flops}
+    fb_s = acct.flops_bytes(cfg, n_spec)
+    fb_f = acct.flops_bytes(cfg)
+    sample_flops = {k: fb_s[k][0] * (ccsdt_blocks if k.startswith("ccsdt") else 1) for k in secs}
+    full_flops = {k: fb_f[k][0] * (cfg.blocks if k.startswith("ccsdt") else 1) for k in secs}
     t_equiv = sum(secs[k] / sample_flops[k] * full_flops[k] for k in secs)
     rate = sum(full_flops.values()) / t_equiv / 1e9
     desc = (f"oracle (C, -O2, OpenMP) on {n_spec} of {cfg.n_elem} elements (p={cfg.p}) for local_grad3/"
@@ -148,117 +172,277 @@ def oracle_sample_rate(cfg, n_spec: int = 8192, ccsdt_blocks: int = 1):
     return rate, desc, sum(secs.values()), {k: sample_flops[k] / secs[k] / 1e9 for k in secs}
 
 
-def threads_used():
+def all_cores():
     n = os.environ.get("OMP_NUM_THREADS")
     return int(n) if n else len(os.sched_getaffinity(0))
 
 
-def run_reference(args, cfg, rank):
+def cpu_baseline(cfg, n_spec):
+    """The oracle on all host cores and on one core (Table IV's "1 core" / "OpenMP"
+    columns), with the CPU model."""
+    cores = all_cores()
+    rate, desc, secs, per = oracle_sample(cfg, n_spec=n_spec, threads=cores)
+    rate1, _, secs1, per1 = oracle_sample(cfg, n_spec=max(256, n_spec // 8), threads=1)
+    return {"value": rate, "unit": "GFLOP/s", "cores": cores, "kind": "oracle", "sample": desc,
+            "cores_all": cores, "gflops_all": rate, "gflops_1core": rate1,
+            "sample_1core": f"{max(256, n_spec // 8)} elements per spectral kernel, 1 block per CCSD(T) family",
+            "cpu_model": cpu_model(), "seconds": secs + secs1, "per_kernel_gflops": per,
+            "per_kernel_gflops_1core": per1}
+
+
+def run_reference(args, cfg):
     """--impl reference: the oracle as it stands on the host cores (rank 0 only)."""
-    if rank.rank != 0:
+    rank, world = env_rank()
+    if rank != 0:
         return
+    cores = all_cores()
     for _ in range(args.warmup):
-        oracle_sample_rate(cfg, n_spec=args.ref_elems)
+        oracle_sample(cfg, n_spec=args.ref_elems, threads=cores)
     rates, secs = [], 0.0
+    desc = ""
     for _ in range(args.steps):
-        r, desc, s, _ = oracle_sample_rate(cfg, n_spec=args.ref_elems)
+        r, desc, s, _ = oracle_sample(cfg, n_spec=args.ref_elems, threads=cores)
         rates.append(r)
         secs += s
     value = float(np.mean(rates))
     line = {
-        "impl": "reference", "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": rank.world,
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs / args.steps * 1e3,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": workload_config(cfg, rank.world),
-        "cpu_baseline": {"value": value, "unit": "GFLOP/s", "cores": threads_used(), "kind": "oracle",
-                         "sample": desc},
+        "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic (counter-based splitmix64, seed 2015)",
+        "config": workload_config(cfg, world, args.scaling),
+        "cpu_baseline": {"value": value, "unit": "GFLOP/s", "cores": cores, "kind": "oracle", "sample": desc,
+                         "cpu_model": cpu_model()},
         "e2e": {"value": value, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
 
 
-def workload_config(cfg, world):
+def workload_config(cfg, world, scaling):
+    per = "per GPU" if scaling == "weak" else f"global, sharded over {world} GPU(s)"
     return {
-        "workload": f"BASELINE configs[1] Nekbone local_grad3 p={cfg.p} N={cfg.n_elem}/GPU + the other hot-path rows "
-                    f"on the same batch: sumfact3d (3-D, p={cfg.p}), sumfact2d (N*(p+1) 2-D elements), CCSD(T) "
-                    f"{'+'.join(cfg.families)} 9-variant fused tile {cfg.tile} x {cfg.blocks} blocks/GPU, check scalars",
-        "p": cfg.p, "n_elem_per_gpu": cfg.n_elem, "ccsdt_tile": cfg.tile, "ccsdt_blocks_per_gpu": cfg.blocks,
-        "parallelism": f"elements+blocks sharded, dp{world}",
+        "workload": f"BASELINE configs[1] Nekbone local_grad3 p={cfg.p} N={cfg.n_elem} ({per}) + the other hot-path "
+                    f"rows on the same batch: sumfact3d (3-D, p={cfg.p}), sumfact2d (N*(p+1) 2-D elements), CCSD(T) "
+                    f"{'+'.join(cfg.families)} 9-variant fused tile {cfg.tile} x {cfg.blocks} blocks ({per}), "
+                    "check scalars",
+        "p": cfg.p, "n_elem": cfg.n_elem, "ccsdt_tile": cfg.tile, "ccsdt_blocks": cfg.blocks,
+        "scaling": scaling, "parallelism": f"elements+blocks sharded, dp{world}",
         "l2": "inputs larger than L2 (U alone is %.1f GB > 126 MB)" % (cfg.n_elem * cfg.P1 ** 3 * 8 / 1e9),
     }
 
 
-def measure_e2e(args, step, rank, dev, stream, flops_step):
-    """Same step through the public API with every input copied from pinned host memory
-    each step and the check scalars read back (timed on the device, max over ranks)."""
+# ---------------------------------------------------------------------------- GPU arm
+def pipe_of(name: str, p: int) -> str:
+    """FP64 pipe a kernel runs on (api.cu dispatch): the CCSD(T) TMA kernels and the
+    spectral tensor-core kernels (P1 in {8, 15, 16}) issue DMMA, the rest DFMA."""
+    if name.startswith("ccsdt"):
+        return "dmma"
+    return "dmma" if (p + 1) in (8, 15, 16) else "dfma"
+
+
+def roof(fl, by, t_s, hbm_gbs, f64_tf, pipe):
+    """Roofline fraction of one launch: t_bound / t_measured, bound = max(HBM, FP64)."""
+    t_hbm, t_f64 = by / (hbm_gbs * 1e9), fl / (f64_tf[pipe] * 1e12)
+    bound = "hbm" if t_hbm >= t_f64 else "alu"
+    return {"gflops": fl / t_s / 1e9, "gbs": by / t_s / 1e9, "bound": bound, "pipe": pipe,
+            "frac": (t_hbm if bound == "hbm" else t_f64) / t_s}
+
+
+def time_calls(fn, inner: int, reps: int, stream) -> float:
+    """Median ms per call of `inner` back-to-back calls, `reps` samples (after one warm call)."""
+    fn()
+    torch.cuda.synchronize()
+    out = []
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(inner):
+            fn()
+        e1.record(stream)
+        e1.synchronize()
+        out.append(e0.elapsed_time(e1) / inner)
+    return float(np.median(out))
+
+
+def measure_configs(dev, hbm_gbs, f64_tf, stream):
+    """BASELINE configs 1, 3, 4, 5 as rows: each kernel timed back to back
+    with CUDA events on synthetic device-resident inputs; frac = roofline fraction."""
+    import paper_conf_icpp_nelsonrbhhjn15_b200 as bc
+    import synthetic as syn
+    f64 = torch.float64
+    rows = {}
+
+    # cfg 1: 3-D sumfact p=4, N=64 (latency-bound: 128.6 KB of traffic)
+    P1, N = 5, 64
+    ops = [bc.fill(torch.empty((P1, P1), dtype=f64, device=dev), syn.TID[n]) for n in ("A", "B", "C")]
+    U = bc.fill(torch.empty((N, P1, P1, P1), dtype=f64, device=dev), syn.TID["U"])
+    V = torch.empty_like(U)
+    call = lambda: bc.sumfact3d(*ops, U, out=V)  # noqa: E731
+    ms_call = time_calls(call, 200, 3, stream)
+    g = torch.cuda.CUDAGraph()
+    s = torch.cuda.Stream(dev)
+    s.wait_stream(stream)
+    with torch.cuda.stream(s):
+        call()
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(100):
+                call()
+    stream.wait_stream(s)
+    ms_graph = time_calls(g.replay, 5, 3, stream) / 100
+    fl, by = acct.sumfact3d(P1, N)
+    rows["cfg1_sumfact3d_p4_N64"] = {"us_per_call": ms_call * 1e3, "us_per_call_graph": ms_graph * 1e3,
+                                     **roof(fl, by, ms_graph * 1e-3, hbm_gbs, f64_tf, pipe_of("sumfact3d", 4)),
+                                     "note": "latency-bound: 16 ns of HBM time; frac shown for the graph-amortised call"}
+    del U, V
+
+    # cfg 3 / 4: CCSD(T) per variant and fused, tiles 16 and 24
+    for fam, tiles in (("d1", (16, 24)), ("d2", (16, 24))):
+        for t in tiles:
+            ext = (t,) * 7
+            t3 = bc.fill(torch.empty(t ** 6, dtype=f64, device=dev), 10)
+            t2s = [bc.fill(torch.empty(t ** 4, dtype=f64, device=dev), 20 + v) for v in range(9)]
+            v2s = [bc.fill(torch.empty(t ** 4, dtype=f64, device=dev), 40 + v) for v in range(9)]
+            inner = 20 if t == 16 else 4
+            per = []
+            for v in range(1, 10):
+                ms = time_calls(lambda: bc.ccsdt(fam, v, ext, t3, t2s[v - 1], v2s[v - 1]), inner, 3, stream)
+                fl, by = acct.ccsdt_variants(ext, 1, fam)
+                per.append({"variant": v, "us": ms * 1e3, **roof(fl, by, ms * 1e-3, hbm_gbs, f64_tf, "dmma")})
+            fr = [r["frac"] for r in per]
+            rows[f"cfg{3 if fam == 'd1' else 4}_{fam}_tile{t}_per_variant"] = {
+                "us_min": min(r["us"] for r in per), "us_max": max(r["us"] for r in per),
+                "frac_min": min(fr), "frac_median": float(np.median(fr)), "frac_max": max(fr),
+                "bound": per[0]["bound"], "gflops_median": float(np.median([r["gflops"] for r in per]))}
+            ms = time_calls(lambda: bc.ccsdt_fused(fam, ext, t3, t2s, v2s), max(2, inner // 4), 3, stream)
+            fl, by = acct.ccsdt_variants(ext, 9, fam)
+            rows[f"cfg{3 if fam == 'd1' else 4}_{fam}_tile{t}_fused9"] = {
+                "us": ms * 1e3, **roof(fl, by, ms * 1e-3, hbm_gbs, f64_tf, "dmma")}
+            del t3, t2s, v2s
+
+    # cfg 5: spectral sweep at N = 2^22 (the largest point), 3-D and 2-D, p in {4, 8, 12}
+    N = 1 << 22
+    for p in (4, 8, 12):
+        P1 = p + 1
+        ops = [bc.fill(torch.empty((P1, P1), dtype=f64, device=dev), syn.TID[n]) for n in ("A", "B", "C")]
+        for form in ("3d", "2d"):
+            shape = (N, P1, P1, P1) if form == "3d" else (N, P1, P1)
+            U = bc.fill(torch.empty(shape, dtype=f64, device=dev), syn.TID["U"])
+            V = torch.empty_like(U)
+            if form == "3d":
+                fn = lambda: bc.sumfact3d(*ops, U, out=V)  # noqa: E731
+                fl, by = acct.sumfact3d(P1, N)
+                name = "sumfact3d"
+            else:
+                fn = lambda: bc.sumfact2d(ops[0], ops[1], U, out=V)  # noqa: E731
+                fl, by = acct.sumfact2d(P1, N)
+                name = "sumfact2d"
+            ms = time_calls(fn, 3, 3, stream)
+            rows[f"cfg5_{form}_p{p}_N{N}"] = {"ms": ms, **roof(fl, by, ms * 1e-3, hbm_gbs, f64_tf, pipe_of(name, p))}
+            del U, V
+            torch.cuda.empty_cache()
+    return rows
+
+
+def pcie_bandwidth(dev, stream, nbytes=1 << 30):
+    """Pinned H2D / D2H copy bandwidth (GB/s) on this GPU: the e2e bound's denominators."""
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    out = {}
+    for name, fn in (("h2d", lambda: d.copy_(h, non_blocking=True)), ("d2h", lambda: h.copy_(d, non_blocking=True))):
+        ms = time_calls(fn, 2, 3, stream)
+        out[name] = nbytes / (ms * 1e-3) / 1e9
+    del h, d
+    return out
+
+
+def measure_e2e(args, step, rank, dev, stream, flops_all, ref_checks):
+    """The same step through the public API with every input copied in from pinned host
+    memory and every output (ur, us, ut, V, V2, all t3 blocks, the check scalars) copied
+    back, each step, overlapped by HostPipeline (timed on the device, max over ranks)."""
     from paper_conf_icpp_nelsonrbhhjn15_b200 import dist as bdist
-    ins = step.inputs()
-    host = [torch.empty(t.shape, dtype=t.dtype, pin_memory=True) for t in ins]
-    for h, t in zip(host, ins):
-        h.copy_(t)
-    out_host = torch.empty(2, dtype=torch.float64, pin_memory=True)
-    h2d = sum(t.numel() * t.element_size() for t in ins)
-    torch.cuda.synchronize(dev)
-
-    def e2e_step():
-        for h, t in zip(host, ins):
-            t.copy_(h, non_blocking=True)
-        chk = step.run()
-        out_host.copy_(chk, non_blocking=True)
-
-    e2e_step()
+    from paper_conf_icpp_nelsonrbhhjn15_b200.workload import HostPipeline
+    t0 = time.perf_counter()
+    pipe = HostPipeline(step, chunks=args.e2e_chunks)
+    pin_s = time.perf_counter() - t0
+    bw = pcie_bandwidth(dev, stream)
+    pipe.run()
     torch.cuda.synchronize(dev)
     bdist.barrier()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
+    pipe.fork(stream)
     for _ in range(args.e2e_steps):
-        e2e_step()
+        pipe.run()
+    pipe.join(stream)
     e1.record(stream)
     torch.cuda.synchronize(dev)
-    ems = bdist.max_over_ranks(e0.elapsed_time(e1) / args.e2e_steps, dev)
-    return {"value": flops_step * rank.world / (ems * 1e-3) / 1e9, "unit": "GFLOP/s",
-            "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 16, "ms_per_step": ems,
-            "api": "paper_conf_icpp_nelsonrbhhjn15_b200 (ctypes -> libbarracuda C ABI), pinned host inputs"}
+    ms = bdist.max_over_ranks(e0.elapsed_time(e1) / args.e2e_steps, dev)
+    # results that reached the host: sum V^2 vs the device-resident step's (same inputs and
+    # kernels; reduced per chunk here, so equal to rounding), and the last chunk / t3 block
+    # in the host ring bitwise equal to the device copies
+    rel = abs(pipe.h_chk[0].item() - ref_checks[0].item()) / abs(ref_checks[0].item())
+    a, b = pipe.bounds[-1]
+    ci = len(pipe.bounds) - 1
+    host_ok = all(torch.equal(pipe.h_ring[nm][ci % pipe.out_slots][:b - a], getattr(step, nm)[a:b].cpu())
+                  for nm in ("ur", "us", "ut", "V"))
+    if step.nb:
+        host_ok = host_ok and torch.equal(pipe.h_t3[(step.nb - 1) % len(pipe.h_t3)], step.t3[-1].cpu())
+    t_bound = max(pipe.h2d_bytes / (bw["h2d"] * 1e9), pipe.d2h_bytes / (bw["d2h"] * 1e9))
+    out = {"value": flops_all / (ms * 1e-3) / 1e9, "unit": "GFLOP/s",
+           "h2d_bytes_per_step": int(pipe.h2d_bytes), "d2h_bytes_per_step": int(pipe.d2h_bytes),
+           "ms_per_step": ms, "pcie_gbs": bw, "pcie_bound_ms": t_bound * 1e3,
+           "frac_of_pcie_bound": t_bound * 1e3 / ms, "pinned_setup_s": pin_s,
+           "sumsq_rel_diff_vs_device_step": rel, "host_results_match_device": bool(host_ok),
+           "host_outputs": f"ring of {pipe.out_slots} pinned chunk slots per output", "chunks": args.e2e_chunks,
+           "api": "paper_conf_icpp_nelsonrbhhjn15_b200 (ctypes -> libbarracuda C ABI), pinned host inputs and "
+                  "outputs, H2D / compute / D2H on three streams"}
+    del pipe
+    return out
 
 
-# ---------------------------------------------------------------------------- main arm
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="barracuda", choices=["barracuda", "reference"])
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
     ap.add_argument("--p", type=int, default=12)
     ap.add_argument("--n-elem", type=int, default=262144)
     ap.add_argument("--tile", type=int, default=16)
     ap.add_argument("--blocks", type=int, default=8)
-    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-chunks", type=int, default=16)
     ap.add_argument("--ref-elems", type=int, default=8192)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-configs", action="store_true")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
-
-    from paper_conf_icpp_nelsonrbhhjn15_b200 import dist as bdist
-    from paper_conf_icpp_nelsonrbhhjn15_b200.workload import StepConfig
-
     cfg = StepConfig(p=args.p, n_elem=args.n_elem, tile=args.tile, blocks=args.blocks)
+
     if args.impl == "reference":
-        world = int(os.environ.get("WORLD_SIZE", "1"))
-        rank = bdist.Rank(int(os.environ.get("RANK", "0")), world, int(os.environ.get("LOCAL_RANK", "0")),
-                          torch.device("cpu"))
-        run_reference(args, cfg, rank)
+        run_reference(args, cfg)
         return
 
+    from paper_conf_icpp_nelsonrbhhjn15_b200 import dist as bdist
     rank = bdist.init()
     import paper_conf_icpp_nelsonrbhhjn15_b200 as bc
     from paper_conf_icpp_nelsonrbhhjn15_b200.workload import Step
 
     dev = rank.device
-    step = Step(cfg, rank.rank, rank.world, dev)
     stream = torch.cuda.current_stream(dev)
-    torch.cuda.synchronize(dev)
+    # FP64 roofline denominators, measured live on this GPU (DESIGN.md §4)
+    f64_tf, f64_src = {}, "live probe (bc_probe_fp64): best of 3 launches, 8 CTAs x 512 threads per SM"
+    try:
+        f64_tf = {k: bc.probe_fp64_tflops(k, dev) for k in ("dfma", "dmma")}
+    except Exception as exc:  # noqa: BLE001
+        f64_tf = {"dfma": FP64_NOMINAL_TFLOPS, "dmma": FP64_NOMINAL_TFLOPS}
+        f64_src = f"nominal 148x64x2x1.965 GHz (probe failed: {exc})"
 
+    step = Step(cfg, rank.rank, rank.world, dev, scaling=args.scaling)
+    torch.cuda.synchronize(dev)
     for _ in range(args.warmup):
         step.run()
     torch.cuda.synchronize(dev)
@@ -289,58 +473,62 @@ def main():
     per_kernel_ms = {n: float(np.mean([ev[s][i].elapsed_time(ev[s][i + 1]) for s in range(args.steps)]))
                      for i, n in enumerate(names)}
 
-    flops_step = step.flops_per_step()
-    value = flops_step * rank.world / (ms * 1e-3) / 1e9
+    flops_local = step.flops_per_step()
+    flops_all = bdist.sum_over_ranks(flops_local, dev)
+    value = flops_all / (ms * 1e-3) / 1e9
 
     # ---- roofline of the dominant kernel (largest share of the step)
     hbm_gbs, hbm_src = load_peaks()
     lps = step.launches_per_step()
     kernels = {}
     for n in names:
-        if n.startswith("check"):
+        if n.startswith("check") or not lps[n]:
             continue
         fl, by = step.fb[n]
         t_launch = per_kernel_ms[n] / lps[n] * 1e-3
-        t_hbm, t_f64 = by / (hbm_gbs * 1e9), fl / (FP64_PEAK_TFLOPS * 1e12)
-        bound = "hbm" if t_hbm >= t_f64 else "alu"
-        kernels[n] = {"ms_per_step": per_kernel_ms[n], "launches": lps[n], "gflops": fl / t_launch / 1e9,
-                      "gbs": by / t_launch / 1e9, "bound": bound,
-                      "frac": (by / t_launch / 1e9 / hbm_gbs) if bound == "hbm" else (fl / t_launch / 1e12 / FP64_PEAK_TFLOPS)}
+        kernels[n] = {"ms_per_step": per_kernel_ms[n], "launches": lps[n],
+                      **roof(fl, by, t_launch, hbm_gbs, f64_tf, pipe_of(n, cfg.p))}
     dom = max(kernels, key=lambda n: kernels[n]["ms_per_step"])
     k = kernels[dom]
-    traffic = load_traffic().get(f"{dom}:p{cfg.p}:n{cfg.n_elem}:t{cfg.tile}")
+    traffic = load_traffic().get(f"{dom}:p{cfg.p}:n{step.n}:t{cfg.tile}")
     if k["bound"] == "hbm":
-        roof = {"kernel": dom, "bound": "hbm", "achieved": k["gbs"], "peak": hbm_gbs, "unit": "GB/s",
-                "frac": k["frac"], "traffic": traffic, "peak_source": hbm_src,
-                "algorithmic_bytes_per_launch": step.fb[dom][1]}
+        roofline = {"kernel": dom, "bound": "hbm", "achieved": k["gbs"], "peak": hbm_gbs, "unit": "GB/s",
+                    "frac": k["frac"], "traffic": traffic, "peak_source": hbm_src,
+                    "algorithmic_bytes_per_launch": step.fb[dom][1]}
     else:
-        roof = {"kernel": dom, "bound": "alu", "achieved": k["gflops"] / 1e3, "peak": FP64_PEAK_TFLOPS,
-                "unit": "TFLOP/s", "frac": k["frac"], "traffic": traffic,
-                "peak_source": "FP64 148x64x2x1.965GHz (measured DMMA 37.1 / DFMA 34.2, profiles/fp64_peak_r01.txt)",
-                "algorithmic_flops_per_launch": step.fb[dom][0]}
+        roofline = {"kernel": dom, "bound": "alu", "achieved": k["gflops"] / 1e3, "peak": f64_tf[k["pipe"]],
+                    "unit": "TFLOP/s", "frac": k["frac"], "traffic": traffic,
+                    "peak_source": f"{k['pipe'].upper()} {f64_src}",
+                    "algorithmic_flops_per_launch": step.fb[dom][0]}
 
-    # ---- end to end: host (pinned) inputs copied in every step, check scalars copied out
+    # ---- end to end: pinned host inputs in, every output out, each step (overlapped)
     e2e = None
     if not args.no_e2e:
         try:
-            e2e = measure_e2e(args, step, rank, dev, stream, flops_step)
+            e2e = measure_e2e(args, step, rank, dev, stream, flops_all, step.checks.cpu().clone())
         except (RuntimeError, MemoryError) as exc:  # e.g. pinned host memory exhausted with many ranks
             e2e = {"value": None, "unit": "GFLOP/s", "error": f"{type(exc).__name__}: {str(exc)[:160]}"}
+    clk = clocks.summary()
+    del step
+    torch.cuda.empty_cache()
+
+    configs = None
+    if rank.rank == 0 and rank.world == 1 and not args.no_configs:
+        configs = measure_configs(dev, hbm_gbs, f64_tf, stream)
 
     cpu = None
     if rank.rank == 0 and rank.world == 1 and not args.no_cpu:
-        rate, desc, secs, per = oracle_sample_rate(cfg, n_spec=args.ref_elems)
-        cpu = {"value": rate, "unit": "GFLOP/s", "cores": threads_used(), "kind": "oracle", "sample": desc,
-               "seconds": secs, "per_kernel_gflops": per}
+        cpu = cpu_baseline(cfg, args.ref_elems)
 
     if rank.rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": rank.world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": args.scaling,
             "vs_baseline": None, "dtype": "f64", "data": "synthetic (counter-based splitmix64, seed 2015)",
-            "config": workload_config(cfg, rank.world),
-            "roofline": roof, "kernels": kernels, "gpu_launches": int(launches),
-            "clocks": clocks.summary(), "e2e": e2e, "cpu_baseline": cpu,
+            "config": workload_config(cfg, rank.world, args.scaling),
+            "roofline": roofline, "kernels": kernels, "gpu_launches": int(launches),
+            "fp64_peak_tflops": {**f64_tf, "source": f64_src},
+            "clocks": clk, "e2e": e2e, "configs": configs, "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
     bdist.finalize()

@@ -58,6 +58,14 @@ def lib():
     return _lib
 
 
+def set_threads(n: int) -> None:
+    """OpenMP thread count for subsequent oracle calls from this thread (bench.py times
+    the oracle on all cores and on one core; no effect on results, which do not depend
+    on the thread count)."""
+    lib()
+    ctypes.CDLL("libgomp.so.1").omp_set_num_threads(int(n))
+
+
 def _c(a) -> np.ndarray:
     a = np.ascontiguousarray(a, dtype=np.float64)
     return a

@@ -26,11 +26,9 @@
 //
 // Kernels (dispatch in run_ccsdt / run_ccsdt_triples_energy):
 //   ccsdt_kernel<FAM,BS>        DFMA cube kernel, any shape (fallback)
-//   ccsdt_mma_kernel<FAM>       16-cube FP64 DMMA, cp.async staging (no tensor maps)
 //   ccsdt_tma_kernel<FAM>       16-cube DMMA, warp-specialised TMA ring (fused, tile 16)
 //   ccsdt_tma24_kernel<FAM>     exact 24-cube version (tile 24, fused and single variant)
 //   ccsdt_svs_kernel<FAM,H>     one d1/d2 variant, t3 streamed through registers (16^3 holes)
-//   ccsdt_sv16b_kernel<FAM>     the same with cp.async.bulk plane streaming (option)
 //   ccsdt_s1h_kernel<H> / ccsdt_s1_stream_kernel<RUN>   s1 streams (equal 16/24 holes / any)
 //   ccsdt_triples_energy_kernel / ccsdt_triples24_kernel  f4: 27 variants + energy (16- / 24-cube)
 #include <cuda.h>
@@ -313,243 +311,12 @@ __global__ void __launch_bounds__(CcGeo<BS>::NT) ccsdt_kernel(const CcsdtParams 
     }
 }
 
-// ==================================================================================
-// Tensor-core path (BS = 16, d1/d2): FP64 DMMA mma.sync.m8n8k4 (no tcgen05 f64 kind
-// exists; DMMA reaches the full FP64 rate with 1/8 of DFMA's instruction count,
-// tools/fp64_peak.cu).  Same unit, cube accumulator and class flush as above.
-//   GEMM per variant: C[s][b] += A[s][k] * B[k][b], s = hole pair (256), b = third hole
-//   (16), k chunk KC = 8 (two m8n8k4 k-steps).  8 warps; warp w owns s in [32w, 32w+32)
-//   x all b: 4 x 2 fragments of 8x8 (16 fp64 accumulators per lane).
-//   smem operand layouts are chosen so fragment reads are bank-conflict free:
-//     d1: A = v2 slice stored [k][s] (row stride 260 = 4 mod 16), B = t2 slice [b][k] (12)
-//     d2: A = t2 slice stored [s][k] (row stride 12),             B = v2 slice [b][k] (12)
-//   and every staging copy is a 16-byte cp.async along the global-contiguous axis.
-// ==================================================================================
-template <int FAM>
-struct MmaGeo {
-    static constexpr int BS = 16, SD = 256, BD = 16, KC = 8, NT = 256;
-    static constexpr int NSTAGE = (FAM == FAM_D1) ? 3 : 2;  // keeps 2 CTAs per SM
-    static constexpr int SS_KS = 260;  // [k][s] row stride (d1 A)
-    static constexpr int SS_SK = 12;   // [s][k] row stride (d2 A)
-    static constexpr int SB_BK = 12;   // [b][k] row stride (B)
-    static constexpr int A_ELEMS = (FAM == FAM_D1) ? KC * SS_KS : SD * SS_SK;  // 2080 | 3072
-    static constexpr int B_ELEMS = BD * SB_BK;                                              // 192
-    static constexpr int STAGE = A_ELEMS + B_ELEMS;                                         // even
-    static constexpr int CST = BS + 1;
-    static constexpr int ACC = BS * CST * CST;  // 4624 (even): the stages stay 16B aligned
-    static constexpr size_t SMEM = (size_t)(ACC + NSTAGE * STAGE) * sizeof(double);
-};
-
+// FP64 tensor-core MMA (no tcgen05 f64 kind exists; DMMA reaches the full FP64 rate with
+// 1/8 of DFMA's instruction count, profiles/fp64_peak_r01.txt)
 __device__ __forceinline__ void dmma_8x8x4(double& c0, double& c1, double a, double b) {
     asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
                  : "+d"(c0), "+d"(c1)
                  : "d"(a), "d"(b));
-}
-
-__device__ __forceinline__ void cp_async_16_zfill(void* dst, const void* src, bool valid) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(smem_u32(dst)), "l"(src),
-                 "r"(valid ? 16 : 0));
-}
-
-template <int FAM>
-__global__ void __launch_bounds__(256) ccsdt_mma_kernel(const CcsdtParams P) {
-    using MG = MmaGeo<FAM>;
-    constexpr int BS = MG::BS, KC = MG::KC, NT = MG::NT, CST = MG::CST;
-    extern __shared__ __align__(16) double sm[];
-    double* acc_s = sm;
-    double* stages = sm + MG::ACC;
-
-    const int ncubes = P.ncube[0] * P.ncube[1] * P.ncube[2];
-    const int cube = blockIdx.x % ncubes;
-    const int plane = blockIdx.x / ncubes;
-    int o[3], len[3];
-    o[0] = (cube % P.ncube[0]) * BS;
-    o[1] = ((cube / P.ncube[0]) % P.ncube[1]) * BS;
-    o[2] = (cube / (P.ncube[0] * P.ncube[1])) * BS;
-    for (int q = 0; q < 3; ++q) len[q] = min(BS, P.qe[q] - o[q]);
-    int qv[3];
-    qv[0] = plane % P.qe[3];
-    qv[1] = (plane / P.qe[3]) % P.qe[4];
-    qv[2] = plane / (P.qe[3] * P.qe[4]);
-    // the unit's t3 values seed the accumulator cube (read once, asynchronously, while
-    // the first operand stages stream in); the cube is stored back once at the end
-    const int64_t pbase = (int64_t)P.qe[0] * P.qe[1] * P.qe[2] *
-                          (qv[0] + (int64_t)P.qe[3] * (qv[1] + (int64_t)P.qe[4] * qv[2]));
-    const int nvol = len[0] * len[1] * len[2];
-    for (int i = threadIdx.x; i < nvol; i += NT) {
-        const int q0 = i % len[0], r = i / len[0];
-        const int q1 = r % len[1], q2 = r / len[1];
-        cp_async_8(acc_s + q0 + CST * (q1 + CST * q2),
-                   P.t3 + pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2)));
-    }
-    cp_async_commit();
-
-    const int H1 = P.ext[N_H1], H3 = P.ext[N_H3];
-    const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6];
-    const int K = P.ext[N_K];
-    const int nchunk = (K + KC - 1) / KC;
-    const int nstage = P.nentry * nchunk;
-
-    // ---- per-thread staging plan.  Thread copies 16-byte pairs at fixed hole positions:
-    //   d1 A: (i2, i3) = ((t & 127) >> 3, 2 (t & 7)), k = (t >> 7) + 2 j      (j < 4)
-    //   d2 A: (i1, i2) = ((t >> 2) & 15, (t >> 6) + 4 j), k pair 2 (t & 3)      (j < 4)
-    //   B (t < 64): third hole i = t >> 2, k pair 2 (t & 3)
-    // Hole offsets are computed once per class; a variant adds its particle offset and a
-    // stage its k offset, so each copy is a pointer increment.
-    const int tid = threadIdx.x;
-    const int H2 = P.ext[N_H2];
-    int64_t hA[3][4];      // per class: hole part of the A offsets (or -1: outside the block)
-    int64_t hB[3];
-    for (int c = 0; c < P.ncls; ++c) {
-        const int hp1 = P.hpos[c][0], hp2 = P.hpos[c][1], hp3 = P.hpos[c][2];
-        const int O1 = o[hp1], O2 = o[hp2], O3 = o[hp3];
-        const int L1 = len[hp1], L2 = len[hp2], L3 = len[hp3];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            if constexpr (FAM == FAM_D1) {
-                const int i2 = (tid & 127) >> 3, i3 = (tid & 7) * 2;
-                hA[c][j] = (i3 < L3 && i2 < L2) ? (O3 + i3) + (int64_t)H3 * (O2 + i2) : -1;
-            } else {
-                const int i1 = (tid >> 2) & 15, i2 = (tid >> 6) + 4 * j;
-                hA[c][j] = (i1 < L1 && i2 < L2) ? (int64_t)K * P4 * ((O1 + i1) + (int64_t)H1 * (O2 + i2)) : -1;
-            }
-        }
-        const int ib = tid >> 2;
-        if constexpr (FAM == FAM_D1)
-            hB[c] = (tid < 64 && ib < L1) ? (int64_t)K * P4 * P5 * (O1 + ib) : -1;
-        else
-            hB[c] = (tid < 64 && ib < L3) ? (int64_t)K * (O3 + ib) : -1;
-    }
-    const int kA = (FAM == FAM_D1) ? (tid >> 7) : 2 * (tid & 3);  // k offset of A copy j = 0
-    const int kB = 2 * (tid & 3);
-    const int dstA = (FAM == FAM_D1) ? (tid >> 7) * MG::SS_KS + 2 * (tid & 127)  // s = i3 + 16 i2 = 2 (t & 127)
-                                     : (tid >> 2) * MG::SS_SK + 2 * (tid & 3);
-    const int dstB = (tid >> 2) * MG::SB_BK + 2 * (tid & 3);
-
-    auto issue = [&](int st) {
-        double* A = stages + (st % MG::NSTAGE) * MG::STAGE;
-        double* B = A + MG::A_ELEMS;
-        const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
-        const int c = P.ecls[e];
-        auto pick = [&](int pos) { return pos == 3 ? qv[0] : (pos == 4 ? qv[1] : qv[2]); };
-        const int p4 = pick(P.ppos[e][0]), p5 = pick(P.ppos[e][1]), p6 = pick(P.ppos[e][2]);
-        const double* __restrict__ t2 = P.opA[e];
-        const double* __restrict__ v2 = P.opB[e];
-        if constexpr (FAM == FAM_D1) {
-            // A[k][s] = v2[h3, h2, p6, k]: offset hole + H3 H2 (p6 + P6 k)
-            const int64_t sk = (int64_t)H3 * H2 * P6;
-            const double* base = v2 + (int64_t)H3 * H2 * p6 + sk * (k0 + kA);
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const bool ok = hA[c][j] >= 0 && (k0 + kA + 2 * j) < K;
-                cp_async_16_zfill(A + dstA + 2 * j * MG::SS_KS, base + (ok ? hA[c][j] + 2 * j * sk : 0), ok);
-            }
-            // B[b][k] = t2[k, p4, p5, h1]: offset k + K (p4 + P4 p5) + hole
-            if (tid < 64) {
-                const bool ok = hB[c] >= 0 && (k0 + kB) < K;
-                const double* src = t2 + (ok ? hB[c] + (k0 + kB) + (int64_t)K * (p4 + (int64_t)P4 * p5) : 0);
-                cp_async_16_zfill(B + dstB, src, ok);
-            }
-        } else {
-            // A[s][k] = t2[k, p4, h1, h2]: offset k + K p4 + hole
-            const double* base = t2 + (k0 + kA) + (int64_t)K * p4;
-            const bool kok = (k0 + kA) < K;
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const bool ok = kok && hA[c][j] >= 0;
-                cp_async_16_zfill(A + dstA + 64 * j * MG::SS_SK, base + (ok ? hA[c][j] : 0), ok);
-            }
-            // B[b][k] = v2[k, h3, p6, p5]: offset k + K (h3 + H3 (p6 + P6 p5))
-            if (tid < 64) {
-                const bool ok = hB[c] >= 0 && (k0 + kB) < K;
-                const double* src = v2 + (ok ? hB[c] + (k0 + kB) + (int64_t)K * H3 * (p6 + (int64_t)P6 * p5) : 0);
-                cp_async_16_zfill(B + dstB, src, ok);
-            }
-        }
-    };
-
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int gq = lane >> 2, tq = lane & 3;  // fragment group / thread-in-group
-    const int s_w = warp * 32;
-    double c[4][2][2];
-#pragma unroll
-    for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-        for (int ni = 0; ni < 2; ++ni) c[mi][ni][0] = c[mi][ni][1] = 0.0;
-
-    // prologue: NSTAGE-1 stages in flight
-#pragma unroll
-    for (int st = 0; st < MG::NSTAGE - 1; ++st) {
-        if (st < nstage) issue(st);
-        cp_async_commit();
-    }
-    for (int st = 0; st < nstage; ++st) {
-        cp_async_wait_n<MG::NSTAGE - 2>();  // stage st has landed (for this thread)
-        __syncthreads();                 // ... for all threads; stage st-1's buffer is free
-        if (st + MG::NSTAGE - 1 < nstage) issue(st + MG::NSTAGE - 1);
-        cp_async_commit();
-        const double* A = stages + (st % MG::NSTAGE) * MG::STAGE;
-        const double* B = A + MG::A_ELEMS;
-        const int e = st / nchunk, k0 = (st - e * nchunk) * KC;
-        const uint32_t smask = P.sign[e] < 0 ? 0x80000000u : 0u;
-#pragma unroll
-        for (int ks = 0; ks < KC / 4; ++ks) {
-            const int kk = ks * 4 + tq;
-            double bf[2], af[4];
-#pragma unroll
-            for (int ni = 0; ni < 2; ++ni) bf[ni] = flip_sign(B[(ni * 8 + gq) * MG::SB_BK + kk], smask);
-#pragma unroll
-            for (int mi = 0; mi < 4; ++mi) {
-                const int sidx = s_w + mi * 8 + gq;
-                af[mi] = (FAM == FAM_D1) ? A[kk * MG::SS_KS + sidx] : A[sidx * MG::SS_SK + kk];
-            }
-#pragma unroll
-            for (int mi = 0; mi < 4; ++mi)
-#pragma unroll
-                for (int ni = 0; ni < 2; ++ni) dmma_8x8x4(c[mi][ni][0], c[mi][ni][1], af[mi], bf[ni]);
-        }
-        const bool last_chunk = (k0 + KC >= K);
-        if (last_chunk && (e + 1 == P.nentry || P.ecls[e + 1] != P.ecls[e])) {
-            const int cl = P.ecls[e];
-            const int strq[3] = {1, CST, CST * CST};
-            const int s1 = strq[P.hpos[cl][0]], s2 = strq[P.hpos[cl][1]], s3 = strq[P.hpos[cl][2]];
-#pragma unroll
-            for (int mi = 0; mi < 4; ++mi) {
-                const int sidx = s_w + mi * 8 + gq;
-                const int hi = sidx >> 4, lo = sidx & 15;
-                const int base = (FAM == FAM_D2) ? (lo * s1 + hi * s2) : (lo * s3 + hi * s2);
-                const int sb = (FAM == FAM_D2) ? s3 : s1;
-#pragma unroll
-                for (int ni = 0; ni < 2; ++ni)
-#pragma unroll
-                    for (int j = 0; j < 2; ++j) {
-                        acc_s[base + (ni * 8 + 2 * tq + j) * sb] += c[mi][ni][j];
-                        c[mi][ni][j] = 0.0;
-                    }
-            }
-        }
-    }
-    cp_async_wait_all();  // (only matters when nstage == 0)
-    __syncthreads();
-    for (int i = threadIdx.x; i < nvol; i += NT) {
-        const int q0 = i % len[0], r = i / len[0];
-        const int q1 = r % len[1], q2 = r / len[1];
-        P.t3[pbase + (o[0] + q0) + (int64_t)P.qe[0] * ((o[1] + q1) + (int64_t)P.qe[1] * (o[2] + q2))] =
-            acc_s[q0 + CST * (q1 + CST * q2)];
-    }
-}
-
-template <int FAM>
-static int launch_ccsdt_mma(const CcsdtParams& P, cudaStream_t s) {
-    static bool init = false;
-    if (!init) {
-        cudaFuncSetAttribute(ccsdt_mma_kernel<FAM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)MmaGeo<FAM>::SMEM);
-        init = true;
-    }
-    const int64_t units = (int64_t)P.ncube[0] * P.ncube[1] * P.ncube[2] * P.qe[3] * P.qe[4] * P.qe[5];
-    if (units == 0) return BC_OK;
-    ccsdt_mma_kernel<FAM><<<(unsigned)units, MmaGeo<FAM>::NT, MmaGeo<FAM>::SMEM, s>>>(P);
-    return launch_status();
 }
 
 // ==================================================================================
@@ -1864,7 +1631,7 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
     for (int q = 3; q < 6; ++q) P.qe[q] = PP;
     for (int q = 0; q < 3; ++q) P.ncube[q] = (H + 15) / 16;
     // exact 24-cubes (tile 24): the 24-cube kernel (BC_NO_TRIP24: the 16-cube one)
-    const bool c24 = H == 24 && K % 2 == 0 && getenv("BC_NO_TRIP24") == nullptr;
+    const bool c24 = H == 24 && K % 2 == 0;
     P.eps_h = eps_h;
     P.eps_p = eps_p;
     P.ws = ws;
@@ -2326,7 +2093,7 @@ static int launch_ccsdt_s1h(const CcsdtParams& P, cudaStream_t s) {
 
 static int launch_ccsdt_s1_stream(const CcsdtParams& P, cudaStream_t s) {
     const int H = P.ext[N_H1];
-    if (H == P.ext[N_H2] && H == P.ext[N_H3] && getenv("BC_S1_GENERIC") == nullptr) {
+    if (H == P.ext[N_H2] && H == P.ext[N_H3]) {
         if (H == 16) return launch_ccsdt_s1h<16>(P, s);
         if (H == 24) return launch_ccsdt_s1h<24>(P, s);
     }
@@ -2557,223 +2324,9 @@ __global__ void __launch_bounds__(SvGeo<H>::NT, SvGeo<H>::MINB) ccsdt_svs_kernel
     }
 }
 
-// ---- sv16 with the Tensor Memory Accelerator streaming the t3 planes (BC_SV16_BULK=1;
-// measured on par with / slightly below the register-streamed kernel above).
-// One persistent CTA per SM.  Thread 0 keeps SVB_PF planes of bulk copies
-// (cp.async.bulk, 32 KB each, mbarrier completion) in flight into a ring of SVB_NS plane
-// buffers; the threads read their 4 x 4 tile from the buffer, accumulate, write it back,
-// and thread 0 bulk-stores the plane (bulk_group; a buffer is reloaded only after the
-// store that last read it has finished reading).  Memory parallelism no longer depends on
-// registers: ~64 KB of loads plus the stores in flight per SM.  Tile reads/writes are
-// conflict-free: odd-`bo` lanes touch their row's second 16-byte half first.
-constexpr int SVB_NS = 4, SVB_PF = 2;
-
-__device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, int bytes, uint32_t bar) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n"
-                 ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
-}
-__device__ __forceinline__ void bulk_store(void* dst, uint32_t src, int bytes) {
-    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;\n" ::"l"(dst), "r"(src), "r"(bytes)
-                 : "memory");
-}
-__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;\n" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void bulk_wait_read() {
-    asm volatile("cp.async.bulk.wait_group.read %0;\n" ::"n"(N) : "memory");
-}
-__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;\n" ::: "memory"); }
-__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory"); }
-
-template <int FAM>
-__global__ void __launch_bounds__(SV_NT, 1) ccsdt_sv16b_kernel(const __grid_constant__ CcsdtParams P, int nplanes) {
-    extern __shared__ __align__(16) double svsm[];
-    const int K = P.ext[N_K];
-    double* ring = svsm;                          // SVB_NS planes of 4096
-    double* As = ring + SVB_NS * 4096;            // [k][f][x]
-    double* Bs = As + K * SV_PS;                  // SVB_NS buffers of [k][y]
-    uint64_t* bars = reinterpret_cast<uint64_t*>(Bs + SVB_NS * 16 * K);
-    const uint32_t bar0 = smem_u32(bars), ring0 = smem_u32(ring);
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int* hp = P.hpos[0];
-    const int posX = (FAM == FAM_D1) ? hp[2] : hp[1];
-    const int posY = (FAM == FAM_D1) ? hp[0] : hp[2];
-    const int posF = (FAM == FAM_D1) ? hp[1] : hp[0];
-    const bool xfast = posX == 0;
-    const int bq = lane & 3, bo = (lane >> 2) & 3;
-    const int bx = xfast ? bq : bo, by = xfast ? bo : bq;
-    const int f = 2 * warp + (lane >> 4);
-    const int sX = 1 << (4 * posX), sY = 1 << (4 * posY), sF = 1 << (4 * posF);
-    const int rstride = xfast ? sY : sX;
-    const int tbase = 4 * bx * sX + 4 * by * sY + f * sF;
-    const bool sw = bo & 1;                      // odd bo: second 16-byte half first (no bank conflicts)
-    const int h0 = sw ? 2 : 0, h1o = 2 - h0;
-    const int P4 = P.ext[N_P4], P5 = P.ext[N_P5], P6 = P.ext[N_P6];
-    const int PO1 = (FAM == FAM_D1) ? P5 : P6, PO2 = (FAM == FAM_D1) ? P4 : P5;
-    auto qstride = [&](int pos) {
-        return pos == 3 ? 4096LL : (pos == 4 ? 4096LL * P.qe[3] : 4096LL * P.qe[3] * P.qe[4]);
-    };
-    const int64_t sp4 = qstride(P.ppos[0][0]), sp5 = qstride(P.ppos[0][1]), sp6 = qstride(P.ppos[0][2]);
-    const double sg = P.sign[0];
-    const double* __restrict__ opA = P.opA[0];
-    const double* __restrict__ opB = P.opB[0];
-    const int lo = (int)((int64_t)nplanes * blockIdx.x / gridDim.x);
-    const int hi = (int)((int64_t)nplanes * (blockIdx.x + 1) / gridDim.x);
-    const int n = hi - lo;
-    auto names = [&](int j, int& a, int& o1, int& o2) {
-        a = j / (PO1 * PO2);
-        const int r = j - a * (PO1 * PO2);
-        o1 = r / PO2;
-        o2 = r - o1 * PO2;
-    };
-    auto plane_ptr = [&](int j) {
-        int a, o1, o2;
-        names(j, a, o1, o2);
-        const int p4 = (FAM == FAM_D1) ? o2 : a, p5 = (FAM == FAM_D1) ? o1 : o2, p6 = (FAM == FAM_D1) ? a : o1;
-        return P.t3 + p4 * sp4 + p5 * sp5 + p6 * sp6;
-    };
-    auto issue_B = [&](int j, double* dst) {
-        int a, o1, o2;
-        names(j, a, o1, o2);
-        const double* src = (FAM == FAM_D1) ? opA + (int64_t)K * (o2 + (int64_t)P4 * o1)
-                                            : opB + (int64_t)K * 16 * (o1 + (int64_t)P6 * o2);
-        const int stride_y = (FAM == FAM_D1) ? K * P4 * P5 : K;
-        for (int i = tid; i < 16 * K; i += SV_NT) {
-            const int y = i / K, k = i - y * K;
-            cp_async_8(dst + k * 16 + y, src + (int64_t)stride_y * y + k);
-        }
-    };
-    if (n <= 0) return;
-    if (tid == 0) {
-        for (int i = 0; i < SVB_NS; ++i) mbar_init(bar0 + 8 * i, 1);
-        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-    }
-    __syncthreads();
-    // prologue: t3 planes lo .. lo+PF-1 (bulk) and their B slices (one cp.async group each)
-    for (int i = 0; i < SVB_PF; ++i) {
-        if (i < n) {
-            if (tid == 0) {
-                mbar_expect_tx(bar0 + 8 * i, 32768);
-                bulk_load(ring0 + i * 32768, plane_ptr(lo + i), 32768, bar0 + 8 * i);
-            }
-            issue_B(lo + i, Bs + i * 16 * K);
-        }
-        cp_async_commit();
-    }
-    int curA = -1;
-    for (int idx = 0; idx < n; ++idx) {
-        const int j = lo + idx, s = idx % SVB_NS;
-        int a, o1, o2;
-        names(j, a, o1, o2);
-        if (a != curA) {  // stage A (sign folded) — once or twice per CTA
-            __syncthreads();
-            if (FAM == FAM_D1) {  // As[k][h2][h3] = v2[h3,h2,p6,k]: 16-byte copies
-                const double* src = opB + 256LL * a;
-                for (int i = tid; i < 128 * K; i += SV_NT) {
-                    const int k = i >> 7, r = 2 * (i & 127);
-                    cp_async_16(As + k * SV_PS + (r >> 4) * SV_RS + (r & 15), src + (int64_t)256 * P6 * k + r);
-                }
-            } else {  // As[k][h1][h2] = t2[k,p4,h1,h2]
-                const double* src = opA + (int64_t)K * a;
-                for (int i = tid; i < 256 * K; i += SV_NT) {
-                    const int r = i / K, k = i - r * K;
-                    cp_async_8(As + k * SV_PS + (r & 15) * SV_RS + (r >> 4), src + (int64_t)K * P4 * r + k);
-                }
-            }
-            cp_async_commit();
-            cp_async_wait_n<0>();
-            if (sg < 0.0) {  // fold the sign into A (exact)
-                __syncthreads();
-                for (int i = tid; i < 256 * K; i += SV_NT) {
-                    double& v = As[(i >> 8) * SV_PS + ((i & 255) >> 4) * SV_RS + (i & 15)];
-                    v = -v;
-                }
-            }
-            curA = a;
-        }
-        cp_async_wait_n<SVB_PF - 1>();                 // this thread's B(j) copies landed
-        mbar_wait(bar0 + 8 * s, (idx / SVB_NS) & 1);   // t3 plane j landed
-        __syncthreads();                               // all B(j), A visible
-        // refill: plane j+PF into the buffer plane j+PF-NS used (its store has read it)
-        if (idx + SVB_PF < n) {
-            const int s2 = (idx + SVB_PF) % SVB_NS;
-            if (tid == 0) {
-                bulk_wait_read<SVB_NS - SVB_PF - 1>();
-                fence_proxy_async();
-                mbar_expect_tx(bar0 + 8 * s2, 32768);
-                bulk_load(ring0 + s2 * 32768, plane_ptr(j + SVB_PF), 32768, bar0 + 8 * s2);
-            }
-            issue_B(j + SVB_PF, Bs + s2 * 16 * K);
-        }
-        cp_async_commit();
-        double* buf = ring + s * 4096 + tbase;
-        double acc[4][4];
-#pragma unroll
-        for (int r = 0; r < 4; ++r) {
-            const double2 u = *reinterpret_cast<const double2*>(buf + r * rstride + h0);
-            const double2 w = *reinterpret_cast<const double2*>(buf + r * rstride + h1o);
-            acc[r][0] = sw ? w.x : u.x;
-            acc[r][1] = sw ? w.y : u.y;
-            acc[r][2] = sw ? u.x : w.x;
-            acc[r][3] = sw ? u.y : w.y;
-        }
-        const double* Ap = As + f * SV_RS + 4 * bx;
-        const double* Bp = Bs + s * 16 * K + 4 * by;
-#pragma unroll 4
-        for (int k = 0; k < K; ++k) {
-            const double2 a01 = *reinterpret_cast<const double2*>(Ap + k * SV_PS);
-            const double2 a23 = *reinterpret_cast<const double2*>(Ap + k * SV_PS + 2);
-            const double2 b01 = *reinterpret_cast<const double2*>(Bp + k * 16);
-            const double2 b23 = *reinterpret_cast<const double2*>(Bp + k * 16 + 2);
-            const double av[4] = {a01.x, a01.y, a23.x, a23.y}, bv[4] = {b01.x, b01.y, b23.x, b23.y};
-#pragma unroll
-            for (int i = 0; i < 4; ++i)
-#pragma unroll
-                for (int jj = 0; jj < 4; ++jj) {
-                    double& t = xfast ? acc[jj][i] : acc[i][jj];
-                    t = fma(av[i], bv[jj], t);
-                }
-        }
-#pragma unroll
-        for (int r = 0; r < 4; ++r) {
-            *reinterpret_cast<double2*>(buf + r * rstride + h0) =
-                sw ? make_double2(acc[r][2], acc[r][3]) : make_double2(acc[r][0], acc[r][1]);
-            *reinterpret_cast<double2*>(buf + r * rstride + h1o) =
-                sw ? make_double2(acc[r][0], acc[r][1]) : make_double2(acc[r][2], acc[r][3]);
-        }
-        fence_proxy_async();  // generic-proxy writes -> visible to the bulk store
-        __syncthreads();
-        if (tid == 0) {
-            bulk_store(plane_ptr(j), ring0 + s * 32768, 32768);
-            bulk_commit();
-        }
-    }
-    if (tid == 0) bulk_wait_all();
-}
-
-template <int FAM>
-static int launch_ccsdt_sv16b(const CcsdtParams& P, cudaStream_t s) {
-    const int K = P.ext[N_K];
-    const size_t smem = ((size_t)SVB_NS * 4096 + (size_t)K * SV_PS + (size_t)SVB_NS * 16 * K) * 8 + SVB_NS * 8;
-    if (smem > 227 * 1024) return 1;
-    const int nplanes = P.qe[3] * P.qe[4] * P.qe[5];
-    if (nplanes == 0) return BC_OK;
-    static bool init = false;
-    if (!init) {
-        cudaFuncSetAttribute(ccsdt_sv16b_kernel<FAM>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-        init = true;
-    }
-    const int grid = nplanes < num_sms() ? nplanes : num_sms();
-    ccsdt_sv16b_kernel<FAM><<<grid, SV_NT, smem, s>>>(P, nplanes);
-    return launch_status();
-}
-
 template <int FAM, int H>
 static int launch_ccsdt_svs(const CcsdtParams& P, cudaStream_t s) {
     using G = SvGeo<H>;
-    if (H == 16 && getenv("BC_SV16_BULK") != nullptr) {
-        const int st = launch_ccsdt_sv16b<FAM>(P, s);
-        if (st != 1) return st;
-    }
     const int K = P.ext[N_K];
     const size_t smem = ((size_t)K * G::PS + 2 * (size_t)H * K) * 8;
     const int nunits = P.qe[3] * P.qe[4] * P.qe[5] * G::NFR;
@@ -2854,26 +2407,20 @@ int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const
     }
     P.nentry = n;
     P.ncls = ncls;
-    if (fam == FAM_S1 && getenv("BC_NO_S1STREAM") == nullptr) {
+    if (fam == FAM_S1) {
         const int st = launch_ccsdt_s1_stream(P, s);
         if (st != 1) return st;  // 1: factors exceed shared memory (cube kernel below)
     }
-    // one d1/d2 variant on 16^3 hole volumes: t3 streamed through registers (HBM-bound).
-    // 24^3 (BC_SVS24=1) measured slower than the 24-cube TMA kernel (0.44 vs 0.51 of HBM).
-    const bool svs_h = ext7[N_H1] == 16 || (ext7[N_H1] == 24 && getenv("BC_SVS24") != nullptr);
-    if (n == 1 && fam != FAM_S1 && ext7[N_H1] == ext7[N_H2] && ext7[N_H2] == ext7[N_H3] && ext7[N_K] <= 32 &&
-        svs_h && getenv("BC_NO_SV16") == nullptr) {
-        if (ext7[N_H1] == 16)
-            return fam == FAM_D1 ? launch_ccsdt_svs<FAM_D1, 16>(P, s) : launch_ccsdt_svs<FAM_D2, 16>(P, s);
-        return fam == FAM_D1 ? launch_ccsdt_svs<FAM_D1, 24>(P, s) : launch_ccsdt_svs<FAM_D2, 24>(P, s);
-    }
+    // one d1/d2 variant on 16^3 hole volumes: t3 streamed through registers (HBM-bound)
+    if (n == 1 && fam != FAM_S1 && ext7[N_H1] == 16 && ext7[N_H2] == 16 && ext7[N_H3] == 16 && ext7[N_K] <= 32)
+        return fam == FAM_D1 ? launch_ccsdt_svs<FAM_D1, 16>(P, s) : launch_ccsdt_svs<FAM_D2, 16>(P, s);
     // tensor-core path: 16-cubes with 16-byte-aligned operand rows (even k, even h3 for d1).
     // It also takes hole extents the 16-cube does not divide (e.g. tile 24 = 16 + 8, ragged
     // cubes zero-filled by TMA): measured 2x faster than the 12-cube DFMA kernel at tile 24.
     const bool tc_shape = (fam != FAM_S1) && (ext7[N_K] % 2 == 0) && (fam != FAM_D1 || ext7[N_H3] % 2 == 0) &&
-                          P.qe[0] >= 12 && P.qe[1] >= 12 && P.qe[2] >= 12 && getenv("BC_NO_MMA") == nullptr;
+                          P.qe[0] >= 12 && P.qe[1] >= 12 && P.qe[2] >= 12;
     // 24-cube TMA path when its padded hole volume is smaller than the 16-cube's (tile 24)
-    if (tc_shape && getenv("BC_NO_TMA") == nullptr && getenv("BC_NO_TMA24") == nullptr) {
+    if (tc_shape) {
         long v16 = 1, v24 = 1;
         for (int q = 0; q < 3; ++q) {
             v16 *= (long)((P.qe[q] + 15) / 16) * 16;
@@ -2885,16 +2432,14 @@ int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const
             if (st != 1) return st;
         }
     }
+    // 16-cube TMA kernel; if the driver cannot encode tensor maps (returns 1), the DFMA
+    // cube kernel below takes the shape
     const int bs = tc_shape ? 16 : choose_bs(P.qe);
     for (int q = 0; q < 3; ++q) P.ncube[q] = (P.qe[q] + bs - 1) / bs;
-    const bool mma_ok = bs == 16 && tc_shape;
-    const bool tma_ok = mma_ok && getenv("BC_NO_TMA") == nullptr;
-    if (tma_ok) {
-        const int st = (fam == FAM_D1) ? launch_ccsdt_tma<FAM_D1>(P, s) : (fam == FAM_D2 ? launch_ccsdt_tma<FAM_D2>(P, s) : 1);
-        if (st != 1) return st;  // 1: tensor maps unavailable
+    if (tc_shape) {
+        const int st = (fam == FAM_D1) ? launch_ccsdt_tma<FAM_D1>(P, s) : launch_ccsdt_tma<FAM_D2>(P, s);
+        if (st != 1) return st;
     }
-    if (mma_ok && fam == FAM_D1) return launch_ccsdt_mma<FAM_D1>(P, s);
-    if (mma_ok && fam == FAM_D2) return launch_ccsdt_mma<FAM_D2>(P, s);
 #define LAUNCH(F)                                                          \
     if (bs == 16) return launch_ccsdt_bs<F, 16>(P, s);                      \
     if (bs == 12) return launch_ccsdt_bs<F, 12>(P, s);                      \

@@ -11,6 +11,7 @@
 // shared-memory wavefront feeds 2R FMAs.  Intermediates never leave shared memory
 // (fusion); only U in and the outputs touch HBM.
 #include <algorithm>
+#include <mutex>
 
 #include "common.cuh"
 
@@ -340,9 +341,6 @@ enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
 #define BC_SMALL_R 3  // sumfact3d lines per thread at P1 < 10 (measured: p=4 0.57 -> 0.65, p=5 0.56 -> 0.62,
                       // p=8 0.47 -> 0.53 of HBM vs R = 2; local_grad3 stays at R = 2)
 #endif
-#ifndef BC_LG3_DIRECT_UR
-#define BC_LG3_DIRECT_UR 0  // local_grad3: store ur from registers instead of in place + copy-out
-#endif
 #ifndef BC_E13_SF2
 #define BC_E13_SF2 0  // sumfact2d elements per group at P1 = 13 (0: derived, 12)
 #endif
@@ -364,6 +362,21 @@ enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
 #ifndef AXE_PB
 #define AXE_PB 4  // ax_e: points per thread whose 6 geometric factors are loaded together
 #endif
+#ifndef BC_CST_R
+#define BC_CST_R 0  // lines per thread of the constant-bank-operator kernels (0: as the smem ones)
+#endif
+#ifndef BC_CST_NUNROLL
+#define BC_CST_NUNROLL 2  // unroll of the constant-operator stages' n loop (measured: 2 >= 1)
+#endif
+#ifndef BC_CST_PF
+#define BC_CST_PF -1  // constant-bank-operator kernels: -1 = prefetch as the smem table, 0/1 = off/on
+#endif
+#ifndef BC_CST_E
+#define BC_CST_E 0  // constant-bank-operator kernels at P1 >= 10: elements per group (0: as the smem table)
+#endif
+#ifndef BC_CST_REGS
+#define BC_CST_REGS 0  // register cap of the constant-bank-operator kernels (0: none)
+#endif
 #ifndef BC_SF2_UNROLL
 #define BC_SF2_UNROLL 1
 #endif
@@ -380,28 +393,36 @@ struct SpecTable {
     // forced elements per group (0: derived from BUF_KB): P1 = 13: 3 x 169 = 507 lines on
     // 128 threads x R = 4 (1% idle lanes instead of 12% with E = 2 on 96 threads)
     static constexpr int EF = (SF3LG3 && P1 == 13) ? BC_E13 : ((KIND == K_SF2 && P1 == 13) ? BC_E13_SF2 : 0);
+    // lines per thread with constant-bank operators (tools/sweep_spectral.py, DESIGN.md
+    // §4.1): 4, except sumfact2d at P1 >= 12 (2)
+    static constexpr int RC = BC_CST_R ? BC_CST_R : ((KIND == K_SF2 && P1 >= 12) ? 2 : 4);
     // unroll of the contracted-index loop: sumfact2d fully (its two stages fit the registers)
     static constexpr int UNROLL = (KIND == K_SF2 && BC_SF2_UNROLL && P1 >= 9) ? P1 : BC_NUNROLL;
 };
 
-template <int P1, int NA, typename T, int NBUF_FIELDS, int KIND = K_SF3>
+template <int P1, int NA, typename T, int NBUF_FIELDS, int KIND = K_SF3, bool CST = false>
 struct Cfg {
     using G = Geo<P1, NA, T>;
     using TB = SpecTable<P1, KIND>;
-    static constexpr bool PREFETCH = TB::PREFETCH && NBUF_FIELDS == 1;  // single-field kernels only
+    static constexpr bool PREFETCH = ((CST && BC_CST_PF >= 0) ? (bool)BC_CST_PF : TB::PREFETCH) &&
+                                     NBUF_FIELDS == 1;  // single-field kernels only
     static constexpr int NBUF = NBUF_FIELDS + (PREFETCH ? 1 : 0);
     static constexpr int BUF_BYTES = TB::BUF_KB * 1024;  // target bytes per element-group buffer
     static constexpr int E0 = BUF_BYTES / (G::ES * (int)sizeof(T));
     // even by default; a measured table entry may force E (odd E x odd P1 groups start 8 bytes
     // off a 16-byte boundary, handled by load_group_async)
-    static constexpr int E = TB::EF ? TB::EF : (E0 < 2 ? 1 : (E0 & ~1));
-    static constexpr int R = TB::R;
+    static constexpr int E = (CST && BC_CST_E && P1 >= 10) ? BC_CST_E : (TB::EF ? TB::EF : (E0 < 2 ? 1 : (E0 & ~1)));
+    static constexpr int R = CST ? TB::RC : TB::R;
     static constexpr int LINES = E * NA * P1;  // lines per axis per group (E * NPTS / P1)
     static constexpr int NT0 = ((LINES + R - 1) / R + 31) / 32 * 32;
     static constexpr int NT = NT0 < 64 ? 64 : (NT0 > 512 ? 512 : NT0);
     static constexpr int VEC = 16 / (int)sizeof(T);
     static constexpr int BUF = (E * G::ES + VEC - 1) / VEC * VEC + VEC;  // + slack for a shifted group
     static constexpr size_t SMEM = (size_t)NBUF * BUF * sizeof(T) + 2 * op_elems<P1, T>() * sizeof(T);
+    // CTAs per SM requested from ptxas (__launch_bounds__): with constant-bank operators
+    // a register cap makes ptxas re-load operators (LDCU) instead of parking them in
+    // registers across the group loop
+    static constexpr int MINB = (CST && BC_CST_REGS) ? (65536 / (NT * BC_CST_REGS) > 0 ? 65536 / (NT * BC_CST_REGS) : 1) : 1;
 };
 
 template <typename KernelT>
@@ -455,6 +476,117 @@ __device__ __forceinline__ void group_loop(int64_t N, const T* __restrict__ src,
     }
 }
 
+// ---------------------------------------------------------------- constant-bank operators
+// For batches of at least OPS_CONST_MIN_N elements the (p+1)x(p+1) operators are staged
+// into the constant bank (c_ops, row-major M[k][n] = cop[k * P1 + n]) by a stream-ordered
+// device-to-device copy ahead of the launch, and the DFMAs read them as uniform-register
+// operands: a warp-wide 16-byte broadcast read from shared memory costs the same 4
+// wavefronts as a full 512-byte read, so with shared-memory operators the SMEM pipe,
+// not the FP64 pipe, bounded these kernels (~1 wavefront per DFMA).
+// OPS_SLOTS slots are reused round robin; a call waits (cudaStreamWaitEvent) for the last
+// kernel that read its slot, so concurrent calls on different streams stay correct.  The
+// slot is a template parameter of the kernels: the operator offsets must be immediates.
+// Small batches keep the shared-memory operators (no extra copy latency).
+constexpr int OPS_SLOTS = 2, OPS_PER_SLOT = 3, OPS_STRIDE = 256;  // 2 x 3 x 16 x 16 doubles = 12 KiB
+#ifndef BC_OPS_CONST_MIN_N
+#define BC_OPS_CONST_MIN_N 128
+#endif
+constexpr int64_t OPS_CONST_MIN_N = BC_OPS_CONST_MIN_N;
+__constant__ double c_ops[OPS_SLOTS][OPS_PER_SLOT][OPS_STRIDE];
+
+int op_slot_acquire(cudaStream_t s, const double* const* ops, int nops, int P1, int* slot);  // below
+void op_slot_release(cudaStream_t s, int slot);
+
+// One warp chunk (lane owns lines L0 + 32 r, r < RR) of a stage with operator OPI of
+// slot CS from the constant bank: y(L, k) = sum_n M[k][n] x(L, n), ascending n (the same
+// fma sequence as lines_chunk).  The n and k loops are fully unrolled, so every operator
+// read is an immediate constant-bank offset: ptxas turns it into an LDCU into a uniform
+// register that the DFMAs take as an operand.  __noinline__: inlined into the group loop,
+// ptxas hoisted all P1^2 operator values out of the loop into regular registers (255
+// registers + spills at P1 = 13); as a call, each chunk re-reads them (108 registers).
+// OMODE 0: outputs overwrite the line in place in `in` (every read of the line precedes
+// its writes, and a line belongs to one lane).  OMODE 1: outputs go to global memory at
+// gdst + gofs(L, k) (streaming stores); with SQ the sum of their squares is returned.
+template <int P1, int NA, int AXIS, int RR, int CS, int OPI, int OMODE, bool SQ>
+__device__ __noinline__ double chunk_c(double* in, double* __restrict__ gdst, int L0, int nlines) {
+    using LN = Line<P1, NA, AXIS, double>;
+    int base[RR];
+#pragma unroll
+    for (int r = 0; r < RR; ++r) {
+        const int L = L0 + r * 32;
+        base[r] = LN::base(L < nlines ? L : (L0 & ~31));
+    }
+    double acc[P1][RR];
+#pragma unroll
+    for (int k = 0; k < P1; ++k)
+#pragma unroll
+        for (int r = 0; r < RR; ++r) acc[k][r] = 0.0;
+    // x(L, n+1) is loaded while step n's FMAs run; the n loop stays rolled (BC_CST_NUNROLL):
+    // inside this non-inlined call n is warp-uniform, so the operator reads are LDCUs with
+    // a uniform-register index (code size ~1 KB per stage instead of ~16 KB fully unrolled:
+    // the unrolled stages missed the instruction cache, 17% of stall samples)
+    double x[RR];
+#pragma unroll
+    for (int r = 0; r < RR; ++r) x[r] = in[base[r]];
+    constexpr int NUNR = BC_CST_NUNROLL;
+#pragma unroll NUNR
+    for (int n = 0; n < P1; ++n) {
+        double xn[RR];
+        const int nn = n + 1 < P1 ? n + 1 : n;
+#pragma unroll
+        for (int r = 0; r < RR; ++r) xn[r] = in[base[r] + nn * LN::STRIDE];
+#pragma unroll
+        for (int k = 0; k < P1; ++k) {
+            const double o = c_ops[CS][OPI][k * P1 + n];
+#pragma unroll
+            for (int r = 0; r < RR; ++r) acc[k][r] = fma(o, x[r], acc[k][r]);
+        }
+#pragma unroll
+        for (int r = 0; r < RR; ++r) x[r] = xn[r];
+    }
+    double sq[RR];  // one partial per line: independent chains instead of one serial chain
+#pragma unroll
+    for (int r = 0; r < RR; ++r) {
+        sq[r] = 0.0;
+        if (L0 + r * 32 < nlines) {
+#pragma unroll
+            for (int k = 0; k < P1; ++k) {
+                if constexpr (OMODE == 0) {
+                    in[base[r] + k * LN::STRIDE] = acc[k][r];
+                } else {
+                    st_cs(gdst + LN::gofs(L0 + r * 32, k), acc[k][r]);
+                    if constexpr (SQ) sq[r] = fma(acc[k][r], acc[k][r], sq[r]);
+                }
+            }
+        }
+    }
+    double t = 0.0;
+#pragma unroll
+    for (int r = 0; r < RR; ++r) t += sq[r];
+    return t;
+}
+
+// apply_lines with operator OPI of constant slot CS (same warp-chunked line assignment as
+// apply_lines_w); returns this thread's sum of squares of its outputs (SQ) or 0.
+template <int P1, int NA, int AXIS, int R, int NT, int CS, int OPI, int OMODE, bool SQ = false>
+__device__ __forceinline__ double apply_lines_c(double* in, double* gdst, int nlines) {
+    constexpr int NW = NT / 32, CH = 32 * R;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int nfull = nlines / CH;
+    double sq = 0.0;
+    for (int c = warp; c < nfull; c += NW)
+        sq += chunk_c<P1, NA, AXIS, R, CS, OPI, OMODE, SQ>(in, gdst, c * CH + lane, nlines);
+    const int rest = nlines - nfull * CH;
+    if (rest > 0 && warp == nfull % NW) {
+        const int L0 = nfull * CH + lane, rr = (rest + 31) >> 5;
+        if constexpr (R >= 4) if (rr == 4) return sq + chunk_c<P1, NA, AXIS, 4, CS, OPI, OMODE, SQ>(in, gdst, L0, nlines);
+        if constexpr (R >= 3) if (rr == 3) return sq + chunk_c<P1, NA, AXIS, (R >= 3 ? 3 : 1), CS, OPI, OMODE, SQ>(in, gdst, L0, nlines);
+        if constexpr (R >= 2) if (rr == 2) return sq + chunk_c<P1, NA, AXIS, (R >= 2 ? 2 : 1), CS, OPI, OMODE, SQ>(in, gdst, L0, nlines);
+        sq += chunk_c<P1, NA, AXIS, 1, CS, OPI, OMODE, SQ>(in, gdst, L0, nlines);
+    }
+    return sq;
+}
+
 // ====================================================================== sumfact3d
 //   S1 W1[l][m][k] = sum_n A[k][n] U[l][m][n]     (axis 2, P:440 / Fig. 2(b))
 //   S2 W2[l][j][k] = sum_m B[j][m] W1[l][m][k]    (axis 1, P:441 / P:214)
@@ -463,11 +595,12 @@ __device__ __forceinline__ void group_loop(int64_t N, const T* __restrict__ src,
 // (consecutive threads own consecutive (j,k): coalesced).  With ws != nullptr the check
 // scalar sum V^2 (R18) is accumulated in the store epilogue: one partial per
 // CTA in ws[8 + blockIdx.x], reduced in fixed order by check_finalize.
-template <int P1, typename T>
-__global__ void __launch_bounds__(Cfg<P1, P1, T, 1, K_SF3>::NT)
+template <int P1, typename T, int CS>
+__global__ void __launch_bounds__(Cfg<P1, P1, T, 1, K_SF3, (CS >= 0)>::NT, Cfg<P1, P1, T, 1, K_SF3, (CS >= 0)>::MINB)
 sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, const T* __restrict__ C,
                  const T* __restrict__ U, T* __restrict__ V, double* __restrict__ ws) {
-    using CF = Cfg<P1, P1, T, 1, K_SF3>;
+    constexpr bool CST = CS >= 0;
+    using CF = Cfg<P1, P1, T, 1, K_SF3, CST>;
     using G = Geo<P1, P1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -475,127 +608,195 @@ sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, co
     T* opB = opA + op_elems<P1, T>();
     T* opC = opB + op_elems<P1, T>();
     T* buf = opC + op_elems<P1, T>();
-    load_op<P1, T, NT>(opA, A);
-    load_op<P1, T, NT>(opB, B);
-    load_op<P1, T, NT>(opC, C);
+    if constexpr (!CST) {
+        load_op<P1, T, NT>(opA, A);
+        load_op<P1, T, NT>(opB, B);
+        load_op<P1, T, NT>(opC, C);
+    }
     double sq = 0.0;
     group_loop<P1, P1, T, NT, CF::E, CF::BUF, CF::PREFETCH>(N, U, buf, [&](T* in, int64_t e0, int ne) {
         const int nlines = ne * P1 * P1;
-        apply_lines<P1, P1, 2, R, NT>(in, opA, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
-        __syncthreads();
-        apply_lines<P1, P1, 1, R, NT>(in, opB, nlines, [&](int, int base, int k, T v) { in[base + k * G::RS] = v; });
-        __syncthreads();
+        auto s1 = [&](int, int base, int k, T v) { in[base + k] = v; };
+        auto s2 = [&](int, int base, int k, T v) { in[base + k * G::RS] = v; };
         T* Vg = V + e0 * G::NPTS;
-        apply_lines<P1, P1, 0, R, NT>(in, opC, nlines, [&](int L, int, int k, T v) {
+        auto s3 = [&](int L, int, int k, T v) {
             st_cs(Vg + Line<P1, P1, 0, T>::gofs(L, k), v);
             sq = fma((double)v, (double)v, sq);
-        });
+        };
+        if constexpr (CST) {
+            constexpr int C = CST ? CS : 0;
+            apply_lines_c<P1, P1, 2, R, NT, C, 0, 0>(in, nullptr, nlines);
+            __syncthreads();
+            apply_lines_c<P1, P1, 1, R, NT, C, 1, 0>(in, nullptr, nlines);
+            __syncthreads();
+            sq += apply_lines_c<P1, P1, 0, R, NT, C, 2, 1, true>(in, Vg, nlines);
+        } else {
+            apply_lines<P1, P1, 2, R, NT>(in, opA, nlines, s1);
+            __syncthreads();
+            apply_lines<P1, P1, 1, R, NT>(in, opB, nlines, s2);
+            __syncthreads();
+            apply_lines<P1, P1, 0, R, NT>(in, opC, nlines, s3);
+        }
     });
     if (ws != nullptr) block_partial(sq, ws + 8);
 }
 
-template <int P1, typename T>
-int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, double* ws, cudaStream_t s) {
-    using CF = Cfg<P1, P1, T, 1, K_SF3>;
+template <int P1, typename T, int CS>
+int launch_sumfact3d_k(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, double* ws, cudaStream_t s) {
+    using CF = Cfg<P1, P1, T, 1, K_SF3, (CS >= 0)>;
     static int occ = 0;
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const size_t smem = CF::SMEM + op_elems<P1, T>() * sizeof(T);
-    int grid = grid_for(sumfact3d_kernel<P1, T>, CF::NT, smem, ngroups, &occ);
+    int grid = grid_for(sumfact3d_kernel<P1, T, CS>, CF::NT, smem, ngroups, &occ);
     if (ws && grid > CHECK_MAX_PARTIALS) grid = CHECK_MAX_PARTIALS;
-    sumfact3d_kernel<P1, T><<<grid, CF::NT, smem, s>>>(N, A, B, C, U, V, ws);
+    sumfact3d_kernel<P1, T, CS><<<grid, CF::NT, smem, s>>>(N, A, B, C, U, V, ws);
     const int st = launch_status();
+    if (CS >= 0) op_slot_release(s, CS);
     if (st || !ws) return st;
     return run_check_finalize(grid, ws, s);
 }
 
+template <int P1, typename T>
+int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, double* ws, cudaStream_t s) {
+    if constexpr (sizeof(T) == 8) {
+        if (N >= OPS_CONST_MIN_N) {
+            const double* ops[3] = {A, B, C};
+            int slot, st;
+            if ((st = op_slot_acquire(s, ops, 3, P1, &slot))) return st;
+            return slot == 0 ? launch_sumfact3d_k<P1, T, 0>(N, A, B, C, U, V, ws, s)
+                             : launch_sumfact3d_k<P1, T, 1>(N, A, B, C, U, V, ws, s);
+        }
+    }
+    return launch_sumfact3d_k<P1, T, -1>(N, A, B, C, U, V, ws, s);
+}
+
 // ====================================================================== sumfact2d
 //   W[l][j] = sum_m A[j][m] U[l][m]  (rows, in place);  V[i][j] = sum_l B[i][l] W[l][j]
-template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, 1, double, 1, K_SF2>::NT)
+template <int P1, int CS>
+__global__ void __launch_bounds__(Cfg<P1, 1, double, 1, K_SF2, (CS >= 0)>::NT, Cfg<P1, 1, double, 1, K_SF2, (CS >= 0)>::MINB)
 sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restrict__ B,
                  const double* __restrict__ U, double* __restrict__ V) {
     using T = double;
-    using CF = Cfg<P1, 1, T, 1, K_SF2>;
+    constexpr bool CST = CS >= 0;
+    using CF = Cfg<P1, 1, T, 1, K_SF2, CST>;
     using G = Geo<P1, 1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* opA = reinterpret_cast<T*>(smem_raw);
     T* opB = opA + op_elems<P1, T>();
     T* buf = opB + op_elems<P1, T>();
-    load_op<P1, T, NT>(opA, A);
-    load_op<P1, T, NT>(opB, B);
+    if constexpr (!CST) {
+        load_op<P1, T, NT>(opA, A);
+        load_op<P1, T, NT>(opB, B);
+    }
     group_loop<P1, 1, T, NT, CF::E, CF::BUF, CF::PREFETCH>(N, U, buf, [&](T* in, int64_t e0, int ne) {
         const int nlines = ne * P1;
         constexpr int U = CF::TB::UNROLL;
         auto st1 = [&](int, int base, int k, T v) { in[base + k] = v; };
-        apply_lines<P1, 1, 2, R, NT, T, decltype(st1), U>(in, opA, nlines, st1);
-        __syncthreads();
         T* Vg = V + e0 * G::NPTS;
         auto st2 = [&](int L, int, int k, T v) { st_cs(Vg + Line<P1, 1, 1, T>::gofs(L, k), v); };
-        apply_lines<P1, 1, 1, R, NT, T, decltype(st2), U>(in, opB, nlines, st2);
+        if constexpr (CST) {
+            constexpr int C = CST ? CS : 0;
+            apply_lines_c<P1, 1, 2, R, NT, C, 0, 0>(in, nullptr, nlines);
+            __syncthreads();
+            apply_lines_c<P1, 1, 1, R, NT, C, 1, 1>(in, Vg, nlines);
+        } else {
+            apply_lines<P1, 1, 2, R, NT, T, decltype(st1), U>(in, opA, nlines, st1);
+            __syncthreads();
+            apply_lines<P1, 1, 1, R, NT, T, decltype(st2), U>(in, opB, nlines, st2);
+        }
     });
+}
+
+template <int P1, int CS>
+int launch_sumfact2d_k(int64_t N, const double* A, const double* B, const double* U, double* V, cudaStream_t s) {
+    using CF = Cfg<P1, 1, double, 1, K_SF2, (CS >= 0)>;
+    static int occ = 0;
+    const int64_t ngroups = (N + CF::E - 1) / CF::E;
+    const int grid = grid_for(sumfact2d_kernel<P1, CS>, CF::NT, CF::SMEM, ngroups, &occ);
+    sumfact2d_kernel<P1, CS><<<grid, CF::NT, CF::SMEM, s>>>(N, A, B, U, V);
+    const int st = launch_status();
+    if (CS >= 0) op_slot_release(s, CS);
+    return st;
 }
 
 template <int P1>
 int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* U, double* V, cudaStream_t s) {
-    using CF = Cfg<P1, 1, double, 1, K_SF2>;
-    static int occ = 0;
-    const int64_t ngroups = (N + CF::E - 1) / CF::E;
-    const int grid = grid_for(sumfact2d_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
-    sumfact2d_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, A, B, U, V);
-    return launch_status();
+    if (N >= OPS_CONST_MIN_N) {
+        const double* ops[2] = {A, B};
+        int slot, st;
+        if ((st = op_slot_acquire(s, ops, 2, P1, &slot))) return st;
+        return slot == 0 ? launch_sumfact2d_k<P1, 0>(N, A, B, U, V, s) : launch_sumfact2d_k<P1, 1>(N, A, B, U, V, s);
+    }
+    return launch_sumfact2d_k<P1, -1>(N, A, B, U, V, s);
 }
 
 // ====================================================================== local_grad3
 //   ur = D along axis 2 (i), us = D along axis 1 (j), ut = D along axis 0 (k) of U[k][j][i]
 // us and ut are stored from registers (coalesced); ur is formed in place (its rows are
 // strided across threads) and copied out coalesced.
-template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, 1, K_LG3>::NT)
+template <int P1, int CS>
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 1, K_LG3, (CS >= 0)>::NT, Cfg<P1, P1, double, 1, K_LG3, (CS >= 0)>::MINB)
 local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ U,
                    double* __restrict__ ur, double* __restrict__ us, double* __restrict__ ut) {
     using T = double;
-    using CF = Cfg<P1, P1, T, 1, K_LG3>;
+    constexpr bool CST = CS >= 0;
+    using CF = Cfg<P1, P1, T, 1, K_LG3, CST>;
     using G = Geo<P1, P1, T>;
     constexpr int NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* opD = reinterpret_cast<T*>(smem_raw);
     T* buf = opD + 2 * op_elems<P1, T>();
-    load_op<P1, T, NT>(opD, D);
+    if constexpr (!CST) load_op<P1, T, NT>(opD, D);
+    // one stage: the operator along AXIS of the group's lines, from smem or the constant bank
     group_loop<P1, P1, T, NT, CF::E, CF::BUF, CF::PREFETCH>(N, U, buf, [&](T* in, int64_t e0, int ne) {
         const int nlines = ne * P1 * P1;
         const int64_t gbase = e0 * G::NPTS;
-        apply_lines<P1, P1, 1, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
-            st_cs(us + gbase + Line<P1, P1, 1, T>::gofs(L, k), v);
-        });
-        apply_lines<P1, P1, 0, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
-            st_cs(ut + gbase + Line<P1, P1, 0, T>::gofs(L, k), v);
-        });
-        if constexpr (BC_LG3_DIRECT_UR) {
-            // ur rows stored straight from registers (lane-strided 8-byte stores; L2 merges the
-            // partial sectors of a warp's 13 consecutive stores)
-            apply_lines<P1, P1, 2, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
-                st_cs(ur + gbase + Line<P1, P1, 2, T>::gofs(L, k), v);
-            });
+        if constexpr (CST) {
+            constexpr int C = CST ? CS : 0;
+            apply_lines_c<P1, P1, 1, R, NT, C, 0, 1>(in, us + gbase, nlines);
+            apply_lines_c<P1, P1, 0, R, NT, C, 0, 1>(in, ut + gbase, nlines);
+            __syncthreads();
+            apply_lines_c<P1, P1, 2, R, NT, C, 0, 0>(in, nullptr, nlines);
         } else {
+            apply_lines<P1, P1, 1, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
+                st_cs(us + gbase + Line<P1, P1, 1, T>::gofs(L, k), v);
+            });
+            apply_lines<P1, P1, 0, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
+                st_cs(ut + gbase + Line<P1, P1, 0, T>::gofs(L, k), v);
+            });
             __syncthreads();
             apply_lines<P1, P1, 2, R, NT>(in, opD, nlines, [&](int, int base, int k, T v) { in[base + k] = v; });
-            __syncthreads();
-            const int total = ne * G::NPTS;
-            for (int f = threadIdx.x; f < total; f += NT) st_cs(ur + gbase + f, in[smem_index<P1, P1, T>(f)]);
         }
+        __syncthreads();
+        const int total = ne * G::NPTS;
+        for (int f = threadIdx.x; f < total; f += NT) st_cs(ur + gbase + f, in[smem_index<P1, P1, T>(f)]);
     });
+}
+
+template <int P1, int CS>
+int launch_local_grad3_k(int64_t N, const double* D, const double* U, double* ur, double* us, double* ut,
+                         cudaStream_t s) {
+    using CF = Cfg<P1, P1, double, 1, K_LG3, (CS >= 0)>;
+    static int occ = 0;
+    const int64_t ngroups = (N + CF::E - 1) / CF::E;
+    const int grid = grid_for(local_grad3_kernel<P1, CS>, CF::NT, CF::SMEM, ngroups, &occ);
+    local_grad3_kernel<P1, CS><<<grid, CF::NT, CF::SMEM, s>>>(N, D, U, ur, us, ut);
+    const int st = launch_status();
+    if (CS >= 0) op_slot_release(s, CS);
+    return st;
 }
 
 template <int P1>
 int launch_local_grad3(int64_t N, const double* D, const double* U, double* ur, double* us, double* ut,
                        cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, 1, K_LG3>;
-    static int occ = 0;
-    const int64_t ngroups = (N + CF::E - 1) / CF::E;
-    const int grid = grid_for(local_grad3_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
-    local_grad3_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, D, U, ur, us, ut);
-    return launch_status();
+    if (N >= OPS_CONST_MIN_N) {
+        int slot, st;
+        if ((st = op_slot_acquire(s, &D, 1, P1, &slot))) return st;
+        return slot == 0 ? launch_local_grad3_k<P1, 0>(N, D, U, ur, us, ut, s)
+                         : launch_local_grad3_k<P1, 1>(N, D, U, ur, us, ut, s);
+    }
+    return launch_local_grad3_k<P1, -1>(N, D, U, ur, us, ut, s);
 }
 
 // ====================================================================== local_grad3_t
@@ -739,6 +940,61 @@ int launch_ax_e(int64_t N, const double* D, const double* U, const double* Gm, d
     const int grid = grid_for(ax_e_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
     ax_e_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, D, U, Gm, W);
     return launch_status();
+}
+
+// ---------------------------------------------------------------- constant-bank slots (host)
+// One mutex serialises slot hand-out, the operator copies, the launch and the event record,
+// so a slot's event always marks the last kernel that read it.  Per device: the symbol's
+// backing address and one event per slot.  While `s` is being captured into a CUDA graph
+// the cross-call wait/record is skipped (stream order inside the graph still holds; a
+// replayed graph must not run concurrently with other spectral calls on the device).
+namespace {
+constexpr int MAX_DEV = 64;
+struct DevSlots {
+    double* base = nullptr;
+    int next = 0;
+    cudaEvent_t ev[OPS_SLOTS] = {};
+    bool recorded[OPS_SLOTS] = {};
+};
+std::mutex g_ops_mu;
+DevSlots g_ops[MAX_DEV];
+thread_local bool g_ops_capturing = false;
+}  // namespace
+
+int op_slot_acquire(cudaStream_t s, const double* const* ops, int nops, int P1, int* slot) {
+    g_ops_mu.lock();
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e == cudaSuccess && (dev < 0 || dev >= MAX_DEV)) e = cudaErrorInvalidDevice;
+    DevSlots* d = e == cudaSuccess ? &g_ops[dev] : nullptr;
+    if (e == cudaSuccess && !d->base) e = cudaGetSymbolAddress(reinterpret_cast<void**>(&d->base), c_ops);
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    if (e == cudaSuccess) e = cudaStreamIsCapturing(s, &cap);
+    g_ops_capturing = cap != cudaStreamCaptureStatusNone;
+    if (e == cudaSuccess) {
+        *slot = d->next;
+        d->next = (d->next + 1) % OPS_SLOTS;
+        if (!g_ops_capturing && d->recorded[*slot]) e = cudaStreamWaitEvent(s, d->ev[*slot], 0);
+    }
+    for (int i = 0; i < nops && e == cudaSuccess; ++i)
+        e = cudaMemcpyAsync(d->base + ((size_t)*slot * OPS_PER_SLOT + i) * OPS_STRIDE, ops[i],
+                            (size_t)P1 * P1 * sizeof(double), cudaMemcpyDeviceToDevice, s);
+    if (e != cudaSuccess) {
+        set_last_cuda_error(e);
+        g_ops_mu.unlock();
+        return BC_ERR_CUDA;
+    }
+    return BC_OK;  // lock held until op_slot_release
+}
+
+void op_slot_release(cudaStream_t s, int slot) {
+    int dev = 0;
+    if (!g_ops_capturing && cudaGetDevice(&dev) == cudaSuccess) {
+        DevSlots& d = g_ops[dev];
+        if (!d.ev[slot]) cudaEventCreateWithFlags(&d.ev[slot], cudaEventDisableTiming);
+        if (d.ev[slot] && cudaEventRecord(d.ev[slot], s) == cudaSuccess) d.recorded[slot] = true;
+    }
+    g_ops_mu.unlock();
 }
 
 // ---------------------------------------------------------------- P1 dispatch

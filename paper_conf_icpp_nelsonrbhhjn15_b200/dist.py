@@ -97,6 +97,15 @@ def max_over_ranks(x: float, device: torch.device) -> float:
     return x
 
 
+def sum_over_ranks(x: float, device: torch.device) -> float:
+    """SUM of a host scalar over ranks (e.g. the flops each rank's shard performed)."""
+    if dist.is_initialized() and dist.get_world_size() > 1:
+        t = torch.tensor([x], dtype=torch.float64, device=_coll_device(device))
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+    return x
+
+
 def finalize() -> None:
     if dist.is_initialized():
         dist.destroy_process_group()

@@ -25,7 +25,9 @@ def bc():
 
 
 def Ns_for(P1):
-    # elements per CTA group E (Cfg in csrc/spectral.cu): 36 KiB / padded element size, made even
+    # elements per CTA group E (Cfg in csrc/spectral.cu): 36 KiB / padded element size, made even.
+    # N < 128 runs the shared-memory-operator kernels, N >= 128 the constant-bank ones
+    # (OPS_CONST_MIN_N in csrc/spectral.cu): both paths at every P1
     return [1, 2, 3, 37, 130]
 
 
@@ -42,9 +44,9 @@ def test_sumfact3d_integer_bitwise(bc, P1):
         assert np.array_equal(to_host(V), oracle.sumfact3d(A, B, C, U)), f"P1={P1} N={N}"
 
 
+@pytest.mark.parametrize("N", [67, 257])
 @pytest.mark.parametrize("P1", ALL_P1)
-def test_sumfact3d_random_tolerance(bc, P1):
-    N = 67
+def test_sumfact3d_random_tolerance(bc, P1, N):
     A, B, C = (syn.tensor(t, (P1, P1)) for t in (2, 3, 4))
     U = syn.tensor(1, (N, P1, P1, P1))
     Ud = to_dev(U)
@@ -82,7 +84,7 @@ def test_sumfact2d(bc, P1):
 @pytest.mark.parametrize("P1", ALL_P1)
 def test_local_grad3(bc, P1):
     D = syn.tensor(6, (P1, P1), kind=syn.KIND_INT)
-    for N in (1, 3, 37):
+    for N in (1, 3, 37, 130):
         U = syn.tensor(1, (N, P1, P1, P1), kind=syn.KIND_INT)
         Ud = to_dev(U)
         outs = tuple(poisoned_like(Ud) for _ in range(3))
@@ -90,10 +92,11 @@ def test_local_grad3(bc, P1):
         for g, r, name in zip(got, oracle.local_grad3(D, U), ("ur", "us", "ut")):
             assert np.array_equal(to_host(g), r), f"{name} P1={P1} N={N}"
     Dg = syn.gll_derivative(P1 - 1)
-    U = syn.tensor(1, (29, P1, P1, P1))
-    got = bc.local_grad3(to_dev(Dg), to_dev(U))
-    for g, r, b in zip(got, oracle.local_grad3(Dg, U), oracle.local_grad3(abs(Dg), abs(U))):
-        assert_abs_close(to_host(g), r, b, 1e-12, f"local_grad3 P1={P1}")
+    for N in (29, 131):
+        U = syn.tensor(1, (N, P1, P1, P1))
+        got = bc.local_grad3(to_dev(Dg), to_dev(U))
+        for g, r, b in zip(got, oracle.local_grad3(Dg, U), oracle.local_grad3(abs(Dg), abs(U))):
+            assert_abs_close(to_host(g), r, b, 1e-12, f"local_grad3 P1={P1} N={N}")
 
 
 @pytest.mark.parametrize("P1", ALL_P1)

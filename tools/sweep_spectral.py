@@ -10,7 +10,7 @@ import torch  # noqa: E402
 import paper_conf_icpp_nelsonrbhhjn15_b200 as bc  # noqa: E402
 import synthetic as syn  # noqa: E402
 
-HBM = 6541.8
+HBM = 6539.2
 
 
 def timeit(fn, reps=10):
