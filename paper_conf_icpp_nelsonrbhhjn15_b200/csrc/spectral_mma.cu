@@ -109,6 +109,11 @@ __device__ __forceinline__ void mma_stage(const double* buf, const double (&a)[M
 #pragma unroll
                 for (int mf = 0; mf < MF; ++mf) dmma(c[t][mf][0], c[t][mf][1], a[mf][ks], b[t]);
         }
+        // the C fragments below are written (in place) to lines that OTHER lanes of this
+        // warp read as B fragments above: order those reads before these writes explicitly
+        // (the mma.sync data dependence already does in practice, but carries no memory-
+        // model ordering; racecheck flagged it)
+        __syncwarp();
 #pragma unroll
         for (int t = 0; t < 2; ++t)
 #pragma unroll

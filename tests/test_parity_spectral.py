@@ -172,3 +172,36 @@ def test_sumfact3d_fused_check_scalar(bc, P1):
     assert_abs_close(to_host(V), Vr, oracle.sumfact3d(abs(A), abs(B), abs(C), abs(U)), 1e-12, "V")
     ref = oracle.sumsq(Vr)
     assert abs(ws[0].item() - ref) <= 1e-12 * ref
+
+
+def test_constant_bank_operators_two_streams_and_graph(bc):
+    """The constant-bank operator slots (csrc/spectral.cu, N >= 128) under concurrency:
+    calls with DIFFERENT operators queued alternately on two streams, more calls than
+    slots, each result equal (bitwise, integer data) to the oracle with its own operators;
+    then the same calls captured into a CUDA graph and replayed."""
+    P1, N = 13, 160
+    U = syn.tensor(1, (N, P1, P1, P1), kind=syn.KIND_INT)
+    Ud = to_dev(U)
+    ops = [[syn.tensor(200 + 3 * i + j, (P1, P1), kind=syn.KIND_INT) for j in range(3)] for i in range(6)]
+    refs = [oracle.sumfact3d(*o, U) for o in ops]
+    dops = [[to_dev(x) for x in o] for o in ops]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    outs = [poisoned_like(Ud) for _ in ops]
+    torch.cuda.synchronize()
+    for i, (o, out) in enumerate(zip(dops, outs)):
+        with torch.cuda.stream(streams[i % 2]):
+            bc.sumfact3d(*o, Ud, out=out)
+    torch.cuda.synchronize()
+    for i, (out, ref) in enumerate(zip(outs, refs)):
+        assert np.array_equal(to_host(out), ref), f"call {i} (stream {i % 2})"
+    g = torch.cuda.CUDAGraph()
+    gouts = [poisoned_like(Ud) for _ in ops]
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        with torch.cuda.graph(g, stream=s):
+            for o, out in zip(dops, gouts):
+                bc.sumfact3d(*o, Ud, out=out)
+    g.replay()
+    torch.cuda.synchronize()
+    for i, (out, ref) in enumerate(zip(gouts, refs)):
+        assert np.array_equal(to_host(out), ref), f"graph call {i}"

@@ -6,12 +6,14 @@ import paper_conf_icpp_nelsonrbhhjn15_b200 as bc
 import synthetic as syn
 dev = torch.device("cuda")
 f = lambda shape, tid: bc.fill(torch.empty(shape, dtype=torch.float64, device=dev), tid)
-for P1 in (5, 13, 16):
-    U = f((7, P1, P1, P1), 1); A = f((P1, P1), 2)
+# P1 = 8 and 16 take the DMMA spectral kernels; N = 7 the shared-memory-operator kernels,
+# N = 130 the constant-bank-operator kernels
+for P1, N in ((5, 7), (5, 130), (8, 7), (13, 7), (13, 130), (16, 7)):
+    U = f((N, P1, P1, P1), 1); A = f((P1, P1), 2)
     bc.sumfact3d(A, A, A, U); bc.sumfact3d(A, A, A, U, check_ws=torch.empty(1024, dtype=torch.float64, device=dev))
-    bc.sumfact2d(A, A, f((9, P1, P1), 3))
+    bc.sumfact2d(A, A, f((N + 2, P1, P1), 3))
     D = torch.from_numpy(syn.gll_derivative(P1 - 1)).to(dev)
-    r = bc.local_grad3(D, U); bc.local_grad3_t(D, *r); bc.ax_e(D, U, f((7, 6, P1, P1, P1), 11))
+    r = bc.local_grad3(D, U); bc.local_grad3_t(D, *r); bc.ax_e(D, U, f((N, 6, P1, P1, P1), 11))
     U32 = U.float(); bc.sumfact3d(A.float(), A.float(), A.float(), U32)
 for ext in ((16,) * 7, (20, 20, 20, 4, 4, 4, 6), (3, 4, 5, 6, 2, 7, 3)):
     h1, h2, h3, p4, p5, p6, k = ext
