@@ -404,7 +404,7 @@ def measure_e2e(args, step, rank, dev, stream, flops_all, ref_checks):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="barracuda", choices=["barracuda", "reference"])
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])

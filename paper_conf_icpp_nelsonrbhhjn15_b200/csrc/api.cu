@@ -2,6 +2,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdlib>
+#include <atomic>
 #include <mutex>
 
 #include "common.cuh"
@@ -48,16 +49,21 @@ static thread_local int64_t g_launches = 0;
 void set_last_cuda_error(cudaError_t e) { g_last_cuda_error = (int)e; }
 void count_launch(int n) { g_launches += n; }
 
+int current_device() {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= BC_MAX_DEVICES) dev = 0;
+    return dev;
+}
+
 int num_sms() {
-    static std::once_flag once;
-    static int sms = 148;
-    std::call_once(once, [] {
-        int dev = 0, v = 0;
-        if (cudaGetDevice(&dev) == cudaSuccess &&
-            cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && v > 0)
-            sms = v;
-    });
-    return sms;
+    static std::atomic<int> sms[BC_MAX_DEVICES];
+    const int dev = current_device();
+    int v = sms[dev].load(std::memory_order_relaxed);
+    if (v == 0) {
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0) v = 148;
+        sms[dev].store(v, std::memory_order_relaxed);
+    }
+    return v;
 }
 
 // ---------------------------------------------------------------- validation helpers

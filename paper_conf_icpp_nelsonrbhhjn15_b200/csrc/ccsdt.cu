@@ -782,17 +782,15 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
 }
 
 // ---- host: tensor maps (driver entry point, no -lcuda)
-static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
-    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
-    static bool tried = false;
-    if (!tried) {
-        tried = true;
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {  // process-wide driver entry point
+    static const PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
         void* f = nullptr;
         cudaDriverEntryPointQueryResult q;
         if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
             q == cudaDriverEntryPointSuccess)
-            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
-    }
+            return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
+        return (PFN_cuTensorMapEncodeTiled_v12000) nullptr;
+    }();
     return fn;
 }
 
@@ -860,7 +858,10 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
         return launch_status();
     };
     const size_t smem1 = 1024 + (size_t)TmaGeo::STAGE_BYTES + TmaGeo::ACC * 8 + 2 * 8;
-    static int occ = 0, occ1 = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
+    static PerDevice<int> occ1_dev;
+    int& occ1 = occ1_dev.get();
     if (P.nentry == 1 && BC_TC16_SINGLE_NS1) return go(ccsdt_tma_kernel<FAM, 1, 3>, smem1, &occ1);
     return go(ccsdt_tma_kernel<FAM>, TmaGeo::SMEM, &occ);
 }
@@ -1155,7 +1156,8 @@ static int launch_ccsdt_tma24(const CcsdtParams& P, cudaStream_t s) {
         }
         if (!ok) return 1;
     }
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     if (occ == 0) {
         cudaFuncSetAttribute(ccsdt_tma24_kernel<FAM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Tma24Geo::SMEM);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_tma24_kernel<FAM>, Tma24Geo::NT, Tma24Geo::SMEM);
@@ -1698,7 +1700,8 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
     }
     P.ns1 = ns;
     if (c24) {
-        static int occ24 = 0;
+        static PerDevice<int> occ24_dev;
+        int& occ24 = occ24_dev.get();
         if (occ24 == 0) {
             cudaFuncSetAttribute(ccsdt_triples24_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Trip24Geo::SMEM);
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ24, ccsdt_triples24_kernel, Trip24Geo::NT, Trip24Geo::SMEM);
@@ -1713,7 +1716,8 @@ int run_ccsdt_triples_energy(const int* ext7, const double* const* t1, const dou
         if (st) return st;
         return run_check_finalize(grid, ws, s);
     }
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     if (occ == 0) {
         cudaFuncSetAttribute(ccsdt_triples_energy_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TmaGeo::SMEM);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_triples_energy_kernel, TmaGeo::NT, TmaGeo::SMEM);
@@ -2079,7 +2083,8 @@ static int launch_ccsdt_s1h(const CcsdtParams& P, cudaStream_t s) {
     constexpr size_t smem = 2 * 9 * (size_t)(H * (H + 2) + H) * 8;
     const int nplanes = P.qe[3] * P.qe[4] * P.qe[5];
     if (nplanes == 0) return BC_OK;
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     if (occ == 0) {
         cudaFuncSetAttribute(ccsdt_s1h_kernel<H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_s1h_kernel<H>, S1S_NT, smem);
@@ -2114,8 +2119,14 @@ static int launch_ccsdt_s1_stream(const CcsdtParams& P, cudaStream_t s) {
         kern<<<grid, S1S_NT, smem, s>>>(P, nplanes);
         return launch_status();
     };
-    static size_t ls4 = 0, ls1 = 0;
-    static int occ4 = 0, occ1 = 0;
+    static PerDevice<size_t> ls4_dev;
+    size_t& ls4 = ls4_dev.get();
+    static PerDevice<size_t> ls1_dev;
+    size_t& ls1 = ls1_dev.get();
+    static PerDevice<int> occ4_dev;
+    int& occ4 = occ4_dev.get();
+    static PerDevice<int> occ1_dev;
+    int& occ1 = occ1_dev.get();
     return run4 ? go(ccsdt_s1_stream_kernel<4>, &ls4, &occ4) : go(ccsdt_s1_stream_kernel<1>, &ls1, &occ1);
 }
 
@@ -2331,8 +2342,10 @@ static int launch_ccsdt_svs(const CcsdtParams& P, cudaStream_t s) {
     const size_t smem = ((size_t)K * G::PS + 2 * (size_t)H * K) * 8;
     const int nunits = P.qe[3] * P.qe[4] * P.qe[5] * G::NFR;
     if (nunits == 0) return BC_OK;
-    static size_t last_smem = 0;
-    static int occ = 0;
+    static PerDevice<size_t> last_smem_dev;
+    size_t& last_smem = last_smem_dev.get();
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     if (smem != last_smem) {
         cudaFuncSetAttribute(ccsdt_svs_kernel<FAM, H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ccsdt_svs_kernel<FAM, H>, G::NT, smem);
@@ -2364,7 +2377,8 @@ static int choose_bs(const int* qe) {
 template <int FAM, int BS>
 static int launch_ccsdt_bs(const CcsdtParams& P, cudaStream_t s) {
     using TT = CcGeo<BS>;
-    static bool init = false;
+    static PerDevice<bool> init_dev;
+    bool& init = init_dev.get();
     if (!init) {
         cudaFuncSetAttribute(ccsdt_kernel<FAM, BS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TT::SMEM);
         init = true;

@@ -10,7 +10,17 @@ namespace bc {
 // thread-local status plumbing (api.cu)
 void set_last_cuda_error(cudaError_t e);
 void count_launch(int n = 1);
-int num_sms();
+int num_sms();  // of the current device
+
+// Launch attributes (cudaFuncSetAttribute, occupancy) are per device: caches keyed by the
+// current device, so one process may call the library on several GPUs.
+constexpr int BC_MAX_DEVICES = 64;
+int current_device();
+template <typename T>
+struct PerDevice {
+    T v[BC_MAX_DEVICES] = {};
+    T& get() { return v[current_device()]; }
+};
 
 inline int launch_status() {
     cudaError_t e = cudaGetLastError();

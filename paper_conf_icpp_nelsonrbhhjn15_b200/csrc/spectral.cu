@@ -644,7 +644,8 @@ sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, co
 template <int P1, typename T, int CS>
 int launch_sumfact3d_k(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, double* ws, cudaStream_t s) {
     using CF = Cfg<P1, P1, T, 1, K_SF3, (CS >= 0)>;
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const size_t smem = CF::SMEM + op_elems<P1, T>() * sizeof(T);
     int grid = grid_for(sumfact3d_kernel<P1, T, CS>, CF::NT, smem, ngroups, &occ);
@@ -711,7 +712,8 @@ sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restri
 template <int P1, int CS>
 int launch_sumfact2d_k(int64_t N, const double* A, const double* B, const double* U, double* V, cudaStream_t s) {
     using CF = Cfg<P1, 1, double, 1, K_SF2, (CS >= 0)>;
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(sumfact2d_kernel<P1, CS>, CF::NT, CF::SMEM, ngroups, &occ);
     sumfact2d_kernel<P1, CS><<<grid, CF::NT, CF::SMEM, s>>>(N, A, B, U, V);
@@ -778,7 +780,8 @@ template <int P1, int CS>
 int launch_local_grad3_k(int64_t N, const double* D, const double* U, double* ur, double* us, double* ut,
                          cudaStream_t s) {
     using CF = Cfg<P1, P1, double, 1, K_LG3, (CS >= 0)>;
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(local_grad3_kernel<P1, CS>, CF::NT, CF::SMEM, ngroups, &occ);
     local_grad3_kernel<P1, CS><<<grid, CF::NT, CF::SMEM, s>>>(N, D, U, ur, us, ut);
@@ -851,7 +854,8 @@ template <int P1>
 int launch_local_grad3_t(int64_t N, const double* D, const double* ur, const double* us, const double* ut,
                          double* U, cudaStream_t s) {
     using CF = Cfg<P1, P1, double, 3, K_LG3T>;
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(local_grad3_t_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
     local_grad3_t_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, D, ur, us, ut, U);
@@ -935,7 +939,8 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
 template <int P1>
 int launch_ax_e(int64_t N, const double* D, const double* U, const double* Gm, double* W, cudaStream_t s) {
     using CF = Cfg<P1, P1, double, 3, K_AXE>;
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     const int64_t ngroups = (N + CF::E - 1) / CF::E;
     const int grid = grid_for(ax_e_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
     ax_e_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, D, U, Gm, W);

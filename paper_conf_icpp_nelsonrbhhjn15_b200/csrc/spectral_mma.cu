@@ -288,7 +288,8 @@ template <int P1>
 static int launch_sf3d_mma(int64_t N, const double* A, const double* B, const double* C, const double* U, double* V,
                            double* ws, cudaStream_t s) {
     using CF = MCfg<P1, P1>;
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     int grid = mma_grid(sumfact3d_mma_kernel<P1>, CF::SMEM, CF::NT, (N + CF::E - 1) / CF::E, &occ);
     if (ws && grid > CHECK_MAX_PARTIALS) grid = CHECK_MAX_PARTIALS;
     sumfact3d_mma_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, A, B, C, U, V, ws);
@@ -299,7 +300,8 @@ static int launch_sf3d_mma(int64_t N, const double* A, const double* B, const do
 template <int P1>
 static int launch_sf2d_mma(int64_t N, const double* A, const double* B, const double* U, double* V, cudaStream_t s) {
     using CF = MCfg<P1, 1>;
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     const int grid = mma_grid(sumfact2d_mma_kernel<P1>, CF::SMEM, CF::NT, (N + CF::E - 1) / CF::E, &occ);
     sumfact2d_mma_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, A, B, U, V);
     return launch_status();
@@ -308,7 +310,8 @@ template <int P1>
 static int launch_lg3_mma(int64_t N, const double* D, const double* U, double* ur, double* us, double* ut,
                           cudaStream_t s) {
     using CF = MCfg<P1, P1>;
-    static int occ = 0;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
     const int grid = mma_grid(local_grad3_mma_kernel<P1>, CF::SMEM, CF::NT, (N + CF::E - 1) / CF::E, &occ);
     local_grad3_mma_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, D, U, ur, us, ut);
     return launch_status();
