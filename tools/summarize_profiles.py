@@ -88,11 +88,12 @@ for f in sorted(os.listdir(G)):
         kn = {"local_grad3_kernel": "local_grad3", "sumfact3d_kernel": "sumfact3d", "sumfact2d_kernel": "sumfact2d",
               "ccsdt_tma_kernel": "ccsdt_tma"}.get(base, base)
         tb = gb("dram__bytes_read.sum") + gb("dram__bytes_write.sum")
+        n_elem = cfg.get("n_elem", cfg.get("n_elem_per_gpu"))
         if kn == "ccsdt_tma":
-            fam = "d1" if "<1>" in name else "d2"
-            traffic[f"ccsdt_{fam}_fused:p{cfg['p']}:n{cfg['n_elem_per_gpu']}:t{cfg['ccsdt_tile']}"] = tb
+            fam = "d1" if ("<1" in name or "<(int)1" in name) else "d2"
+            traffic[f"ccsdt_{fam}_fused:p{cfg['p']}:n{n_elem}:t{cfg['ccsdt_tile']}"] = tb
         else:
-            traffic[f"{kn}:p{cfg['p']}:n{cfg['n_elem_per_gpu']}:t{cfg['ccsdt_tile']}"] = tb
+            traffic[f"{kn}:p{cfg['p']}:n{n_elem}:t{cfg['ccsdt_tile']}"] = tb
 open(os.path.join(P, f"ncu_summary_{tag}.md"), "w").write("\n".join(lines) + "\n")
 json.dump(traffic, open(os.path.join(P, "traffic.json"), "w"), indent=1)
 subprocess.run(["cp", os.path.join(G, "launches.csv"), os.path.join(P, f"launches_{tag}.csv")])
