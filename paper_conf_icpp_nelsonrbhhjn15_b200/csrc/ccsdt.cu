@@ -524,6 +524,10 @@ __device__ __forceinline__ void tma_flush_class(double* acc_s, double (&c)[4][2]
     const int s1 = hp[0] == 0 ? 1 : (hp[0] == 1 ? CST : CST * CST);
     const int s2 = hp[1] == 0 ? 1 : (hp[1] == 1 ? CST : CST * CST);
     const int s3 = hp[2] == 0 ? 1 : (hp[2] == 1 ? CST : CST * CST);
+    // The 16 positions a thread updates are distinct, but the compiler cannot prove it and
+    // serialised the read-modify-writes (LDS -> DADD -> STS -> next LDS: ~16 dependent
+    // round trips per flush).  All reads are issued first, then the adds and stores.
+    int pos[4][2][2];
 #pragma unroll
     for (int mi = 0; mi < 4; ++mi) {
         int hi, lo;  // strided pair (lo = fast name, hi = h2)
@@ -540,11 +544,24 @@ __device__ __forceinline__ void tma_flush_class(double* acc_s, double (&c)[4][2]
 #pragma unroll
         for (int ni = 0; ni < 2; ++ni)
 #pragma unroll
+            for (int j = 0; j < 2; ++j) pos[mi][ni][j] = rowoff + (ni * 8 + permK(2 * tq + j)) * sb;
+    }
+    double old[4][2][2];
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+        for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
+            for (int j = 0; j < 2; ++j) old[mi][ni][j] = acc_s[pos[mi][ni][j]];
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+        for (int ni = 0; ni < 2; ++ni)
+#pragma unroll
             for (int j = 0; j < 2; ++j) {
-                acc_s[rowoff + (ni * 8 + permK(2 * tq + j)) * sb] += c[mi][ni][j];
+                acc_s[pos[mi][ni][j]] = old[mi][ni][j] + c[mi][ni][j];
                 c[mi][ni][j] = 0.0;
             }
-    }
 }
 
 // NSR: ring depth.  Single-variant launches (one stage per unit at tile 16) use NSR = 1
@@ -1087,11 +1104,16 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
                     const int h2 = 3 * warp + mi / 3;
                     const int lo = 8 * (mi % 3) + ((FAM == FAM_D1) ? gq : perm64(gq));
                     double* row = acc_s + lo * slo + h2 * s2;
+                    double old[3][2];  // reads first (positions are distinct; see tma_flush_class)
+#pragma unroll
+                    for (int ni = 0; ni < 3; ++ni)
+#pragma unroll
+                        for (int j = 0; j < 2; ++j) old[ni][j] = row[(8 * ni + perm64(2 * tq + j)) * sth];
 #pragma unroll
                     for (int ni = 0; ni < 3; ++ni)
 #pragma unroll
                         for (int j = 0; j < 2; ++j) {
-                            row[(8 * ni + perm64(2 * tq + j)) * sth] += c[mi][ni][j];
+                            row[(8 * ni + perm64(2 * tq + j)) * sth] = old[ni][j] + c[mi][ni][j];
                             c[mi][ni][j] = 0.0;
                         }
                 }
@@ -1433,11 +1455,16 @@ __device__ __forceinline__ void t24_flush(double* acc_s, double (&c)[9][3][2], c
         const int h2 = 3 * warp + mi / 3;
         const int lo = 8 * (mi % 3) + ((FE == FAM_D1) ? gq : perm64(gq));
         double* row = acc_s + lo * slo + h2 * s2;
+        double old[3][2];  // reads first (positions are distinct; see tma_flush_class)
+#pragma unroll
+        for (int ni = 0; ni < 3; ++ni)
+#pragma unroll
+            for (int j = 0; j < 2; ++j) old[ni][j] = row[(8 * ni + perm64(2 * tq + j)) * sth];
 #pragma unroll
         for (int ni = 0; ni < 3; ++ni)
 #pragma unroll
             for (int j = 0; j < 2; ++j) {
-                row[(8 * ni + perm64(2 * tq + j)) * sth] += c[mi][ni][j];
+                row[(8 * ni + perm64(2 * tq + j)) * sth] = old[ni][j] + c[mi][ni][j];
                 c[mi][ni][j] = 0.0;
             }
     }
