@@ -9,7 +9,7 @@ import subprocess
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-G = os.path.join(ROOT, "gpurun_out")
+G = os.environ.get("G") or os.path.join(ROOT, "gpurun_out")
 P = os.path.join(ROOT, "profiles")
 tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
 
@@ -31,17 +31,32 @@ hi = [i for i, r in enumerate(rows) if "Kernel Name" in r][0]
 h = rows[hi]
 ki, vi = h.index("Kernel Name"), h.index("Metric Value")
 agg = collections.defaultdict(list)
+setup = collections.defaultdict(list)
 for r in rows[hi + 1:]:
     if len(r) > vi:
         try:
-            agg[r[ki].split("(")[0]].append(float(r[vi].replace(",", "")))
+            name = r[ki].split("(")[0]
+            v = float(r[vi].replace(",", ""))
         except ValueError:
-            pass
+            continue
+        # the step's kernels, template variants merged (the constant-bank slot 0/1
+        # instantiations); setup kernels (FP64 probes, input fills, torch) listed apart
+        if "probe_" in name or "fill_kernel" in name or "at::" in name:
+            setup[name].append(v)
+        else:
+            base = name.replace("void ", "")
+            if "<" in base and ("sumfact" in base or "local_grad3" in base):
+                base = base[:base.rindex(",")] + ">" if base.count(",") else base
+            agg[base].append(v)
 tot = sum(sum(v) for v in agg.values())
 lines += ["", "## ncu launch list (gpu__time_duration, --clock-control none; bench --steps 2 --warmup 3)", "",
+          "Step kernels only (warm-up + timed steps; shares of their total); setup kernels "
+          "(live FP64 probes, input fills) below the table.", "",
           "| kernel | launches | total us | share |", "|---|---|---|---|"]
 for k, v in sorted(agg.items(), key=lambda x: -sum(x[1])):
     lines.append(f"| {k} | {len(v)} | {sum(v)/1e3:.1f} | {sum(v)/tot*100:.1f}% |")
+lines.append("")
+lines.append("setup: " + ", ".join(f"{k} x{len(v)} {sum(v)/1e3:.0f} us" for k, v in setup.items()))
 
 WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "sm__warps_active.avg.pct_of_peak_sustained_active",
