@@ -350,11 +350,18 @@ struct TmaMaps {
 #ifndef BC_TC16_KC
 #define BC_TC16_KC 16
 #endif
+#ifndef BC_TC16_NS
+#define BC_TC16_NS 0  // ring depth of the fused tile-16 kernel (0: 2 at KC = 16, 4 at KC = 8)
+#endif
+#ifndef BC_TC16_MINB
+#define BC_TC16_MINB 2  // CTAs per SM of the fused tile-16 kernel
+#endif
 struct TmaGeo {
     // two CTAs per SM (measured better than one CTA with a deeper ring).  KC = 8: 64 B
     // operand rows (64B swizzle), 4-deep ring;  KC = 16: 128 B rows (128B swizzle, half the
     // TMA rows per byte), 2-deep ring
-    static constexpr int BS = 16, KC = BC_TC16_KC, NS = KC == 16 ? 2 : 4, NCW = 8, NT = (NCW + 1) * 32;
+    static constexpr int BS = 16, KC = BC_TC16_KC, NS = BC_TC16_NS ? BC_TC16_NS : (KC == 16 ? 2 : 4), NCW = 8,
+                         NT = (NCW + 1) * 32;
     static constexpr int A_BYTES = 16 * 16 * KC * 8;  // 16 | 32 KiB
     static constexpr int B_BYTES = 16 * KC * 8;       // 1 | 2 KiB
     static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;  // multiple of 1 KiB
@@ -591,7 +598,7 @@ __device__ __forceinline__ void unit_add(UnitDigits& x, const UnitDigits& s, con
         x.d[i] = carry ? v - r[i] : v;
     }
 }
-template <int FAM, int NSR = TmaGeo::NS, int MINB = 2>
+template <int FAM, int NSR = TmaGeo::NS, int MINB = BC_TC16_MINB>
 __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __grid_constant__ CcsdtParams P,
                                                                      const __grid_constant__ TmaMaps M, int units) {
     using TG = TmaGeo;

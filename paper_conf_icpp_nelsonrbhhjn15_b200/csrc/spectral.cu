@@ -264,6 +264,9 @@ __device__ __forceinline__ void lines_chunk(const T* in, const T* opT, int L0, i
             fmas(x, o, z);
         }
     }
+    // lanes of a ragged chunk read (and discard) the chunk's first line, which lane 0
+    // overwrites in place below: order every lane's reads before the writes
+    __syncwarp();
 #pragma unroll
     for (int r = 0; r < RR; ++r)
         if (L0 + r * 32 < nlines) {
@@ -544,6 +547,7 @@ __device__ __noinline__ double chunk_c(double* in, double* __restrict__ gdst, in
 #pragma unroll
         for (int r = 0; r < RR; ++r) x[r] = xn[r];
     }
+    __syncwarp();  // dummy reads of ragged lanes (the chunk's first line) precede the in-place writes
     double sq[RR];  // one partial per line: independent chains instead of one serial chain
 #pragma unroll
     for (int r = 0; r < RR; ++r) {
