@@ -350,6 +350,9 @@ struct TmaMaps {
 #ifndef BC_TC16_KC
 #define BC_TC16_KC 16
 #endif
+#ifndef BC_FLUSH_ALWAYS_BAR
+#define BC_FLUSH_ALWAYS_BAR 0  // consumer barrier before every class flush (else only where needed)
+#endif
 #ifndef BC_TC16_NS
 #define BC_TC16_NS 0  // ring depth of the fused tile-16 kernel (0: 2 at KC = 16, 4 at KC = 8)
 #endif
@@ -748,7 +751,7 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
                 // needed after the first flush when the class spans more than NS stages: the
                 // producer refills a slot only after all consumers released it, so the
                 // fastest warp is at most NS stages ahead of the slowest.
-                const bool need_bar = !seeded || cls_stages <= NS;
+                const bool need_bar = BC_FLUSH_ALWAYS_BAR || !seeded || cls_stages <= NS;
                 if (!seeded) cp_async_wait_n<0>();
                 seeded = true;
                 if (need_bar) named_bar_sync(1, 256);
@@ -1089,7 +1092,7 @@ __global__ void __launch_bounds__(Tma24Geo::NT, 1) ccsdt_tma24_kernel(const __gr
                 // another is still flushing the previous class: the producer refills a slot
                 // only after all consumers released it, so the fastest warp is at most NS
                 // stages ahead of the slowest.
-                const bool need_bar = !seeded || cls_stages <= NS;
+                const bool need_bar = BC_FLUSH_ALWAYS_BAR || !seeded || cls_stages <= NS;
                 if (!seeded) cp_async_wait_n<0>();
                 seeded = true;
                 if (need_bar) named_bar_sync(1, NCT);
