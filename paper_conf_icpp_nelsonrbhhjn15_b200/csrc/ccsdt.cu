@@ -350,6 +350,12 @@ struct TmaMaps {
 #ifndef BC_TC16_KC
 #define BC_TC16_KC 16
 #endif
+#ifndef BC_EXP16_NOFLUSH
+#define BC_EXP16_NOFLUSH 0  // timing experiments only: skip the class flushes of the 16-cube kernel
+#endif
+#ifndef BC_EXP16_NOSTORE
+#define BC_EXP16_NOSTORE 0  // timing experiments only: skip the store / re-seed of the 16-cube kernel
+#endif
 #ifndef BC_FLUSH_ALWAYS_BAR
 #define BC_FLUSH_ALWAYS_BAR 0  // consumer barrier before every class flush (else only where needed)
 #endif
@@ -756,7 +762,15 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
                 seeded = true;
                 if (need_bar) named_bar_sync(1, 256);
                 cls_stages = 0;
-                tma_flush_class<FAM>(acc_s, c, P.hpos[P.ecls[e_cur]], warp, gq, tq);
+                if (BC_EXP16_NOFLUSH) {  // timing experiment only (wrong results)
+#pragma unroll
+                    for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+                        for (int ni = 0; ni < 2; ++ni)
+                            if (c[mi][ni][0] == 1.2345) acc_s[mi] = c[mi][ni][1];
+                } else {
+                    tma_flush_class<FAM>(acc_s, c, P.hpos[P.ecls[e_cur]], warp, gq, tq);
+                }
             }
             if (last_chunk && e < P.nentry) {
                 smask = P.smask[e];
@@ -767,8 +781,9 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
             cp_async_wait_n<0>();
             seeded = true;
         }
-        named_bar_sync(1, 256);  // all flushes into this cube are done
-        if (full_cubes) {
+        named_bar_sync(1, 256);  // all flushes into / reads of this cube are done
+        if (BC_EXP16_NOSTORE) {  // timing experiment only (wrong results)
+        } else if (full_cubes) {
             // store this unit and seed the CTA's next unit, position by position (same owner)
             const int q0 = tid & 15, q1 = tid >> 4;
             double* dstg = P.t3 + pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)P.qe[1] * o[2]);
