@@ -70,6 +70,18 @@ def ccsdt_variants(ext, nvar: int, family: str = "d1"):
     return 2.0 * n3 * k * nvar, 16.0 * n3 + 8.0 * nvar * nop
 
 
+def triples_energy(ext):
+    """f4: all 27 triples variants (9 s1 + 9 d1 + 9 d2) into a t3 that is never stored,
+    plus the energy epilogue (~4 flops per element beyond the sums); bytes = the operands
+    (t3 neither read nor written)."""
+    h1, h2, h3, p4, p5, p6, k = ext
+    n3 = h1 * h2 * h3 * p4 * p5 * p6
+    fl = ccsdt_variants(ext, 9, "d1")[0] + ccsdt_variants(ext, 9, "d2")[0] + ccsdt_variants(ext, 9, "s1")[0]
+    ops = 9 * ((p4 * h1 + h3 * h2 * p6 * p5) + (k * p4 * p5 * h1 + h3 * h2 * p6 * k) +
+               (k * p4 * h1 * h2 + k * h3 * p6 * p5))
+    return fl + 4.0 * n3, 8.0 * ops
+
+
 def energy(ext):
     """Energy-style check over one t3: ~9 flops per element (denominator + t^2/den)."""
     n3 = 1

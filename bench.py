@@ -320,6 +320,48 @@ def measure_configs(dev, hbm_gbs, f64_tf, stream):
                 "us": ms * 1e3, **roof(fl, by, ms * 1e-3, hbm_gbs, f64_tf, "dmma")}
             del t3, t2s, v2s
 
+    # NEXT rows: f1 local_grad3_t and f2 ax_e at p = 12, f3 s1 fused and
+    # f4 (27 variants + energy, t3 never stored) at tiles 16 and 24
+    p, P1 = 12, 13
+    D = torch.from_numpy(syn.gll_derivative(p)).to(dev)
+    N = 262144
+    fields = [bc.fill(torch.empty((N, P1, P1, P1), dtype=f64, device=dev), 7 + i) for i in range(3)]
+    W = torch.empty_like(fields[0])
+    ms = time_calls(lambda: bc.local_grad3_t(D, *fields, out=W), 3, 3, stream)
+    fl, by = acct.local_grad3_t(P1, N)
+    rows[f"f1_local_grad3_t_p12_N{N}"] = {"ms": ms, **roof(fl, by, ms * 1e-3, hbm_gbs, f64_tf, pipe_of("lg3t", p))}
+    del fields, W
+    torch.cuda.empty_cache()
+    N = 65536
+    U = bc.fill(torch.empty((N, P1, P1, P1), dtype=f64, device=dev), syn.TID["U"])
+    Gm = bc.fill(torch.empty((N, 6, P1, P1, P1), dtype=f64, device=dev), syn.TID["G"])
+    W = torch.empty_like(U)
+    ms = time_calls(lambda: bc.ax_e(D, U, Gm, out=W), 3, 3, stream)
+    fl, by = acct.ax_e(P1, N)
+    rows[f"f2_ax_e_p12_N{N}"] = {"ms": ms, **roof(fl, by, ms * 1e-3, hbm_gbs, f64_tf, pipe_of("ax_e", p))}
+    del U, Gm, W
+    torch.cuda.empty_cache()
+    for t in (16, 24):
+        ext = (t,) * 7
+        t3 = bc.fill(torch.empty(t ** 6, dtype=f64, device=dev), 10)
+        ops = {}
+        for i, fam in enumerate(("s1", "d1", "d2")):
+            na, nb = bc.operand_sizes(fam, ext)
+            ops[fam] = ([bc.fill(torch.empty(na, dtype=f64, device=dev), 100 + 20 * i + v) for v in range(9)],
+                        [bc.fill(torch.empty(nb, dtype=f64, device=dev), 110 + 20 * i + v) for v in range(9)])
+        ms = time_calls(lambda: bc.ccsdt_fused("s1", ext, t3, *ops["s1"]), 8 if t == 16 else 2, 3, stream)
+        fl, by = acct.ccsdt_variants(ext, 9, "s1")
+        rows[f"f3_s1_tile{t}_fused9"] = {"us": ms * 1e3, **roof(fl, by, ms * 1e-3, hbm_gbs, f64_tf, "dfma")}
+        eh = bc.fill(torch.empty(3 * t, dtype=f64, device=dev), syn.TID["EPS_H"], kind=bc.KIND_RANGE, lo=-2.0, hi=-0.5)
+        ep = bc.fill(torch.empty(3 * t, dtype=f64, device=dev), syn.TID["EPS_P"], kind=bc.KIND_RANGE, lo=0.5, hi=2.0)
+        ws = torch.empty(bc.BC_CHECK_WS_DOUBLES, dtype=f64, device=dev)
+        ms = time_calls(lambda: bc.ccsdt_triples_energy(ext, ops["s1"], ops["d1"], ops["d2"], eh, ep, ws),
+                        4 if t == 16 else 1, 3, stream)
+        fl, by = acct.triples_energy(ext)
+        rows[f"f4_triples_energy_tile{t}"] = {"us": ms * 1e3, **roof(fl, by, ms * 1e-3, hbm_gbs, f64_tf, "dmma")}
+        del t3, ops
+        torch.cuda.empty_cache()
+
     # cfg 5: spectral sweep at N = 2^22 (the largest point), 3-D and 2-D, p in {4, 8, 12}
     N = 1 << 22
     for p in (4, 8, 12):

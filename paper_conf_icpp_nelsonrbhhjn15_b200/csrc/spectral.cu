@@ -398,7 +398,8 @@ struct SpecTable {
     static constexpr int EF = (SF3LG3 && P1 == 13) ? BC_E13 : ((KIND == K_SF2 && P1 == 13) ? BC_E13_SF2 : 0);
     // lines per thread with constant-bank operators (tools/sweep_spectral.py, DESIGN.md
     // §4.1): 4, except sumfact2d at P1 >= 12 (2)
-    static constexpr int RC = BC_CST_R ? BC_CST_R : ((KIND == K_SF2 && P1 >= 12) ? 2 : 4);
+    static constexpr int RC = BC_CST_R ? BC_CST_R
+                                       : ((KIND == K_SF2 && P1 >= 12) || KIND == K_LG3T || KIND == K_AXE ? 2 : 4);
     // unroll of the contracted-index loop: sumfact2d fully (its two stages fit the registers)
     static constexpr int UNROLL = (KIND == K_SF2 && BC_SF2_UNROLL && P1 >= 9) ? P1 : BC_NUNROLL;
 };
@@ -502,16 +503,24 @@ void op_slot_release(cudaStream_t s, int slot);
 
 // One warp chunk (lane owns lines L0 + 32 r, r < RR) of a stage with operator OPI of
 // slot CS from the constant bank: y(L, k) = sum_n M[k][n] x(L, n), ascending n (the same
-// fma sequence as lines_chunk).  The n and k loops are fully unrolled, so every operator
-// read is an immediate constant-bank offset: ptxas turns it into an LDCU into a uniform
-// register that the DFMAs take as an operand.  __noinline__: inlined into the group loop,
-// ptxas hoisted all P1^2 operator values out of the loop into regular registers (255
-// registers + spills at P1 = 13); as a call, each chunk re-reads them (108 registers).
-// OMODE 0: outputs overwrite the line in place in `in` (every read of the line precedes
-// its writes, and a line belongs to one lane).  OMODE 1: outputs go to global memory at
-// gdst + gofs(L, k) (streaming stores); with SQ the sum of their squares is returned.
-template <int P1, int NA, int AXIS, int RR, int CS, int OPI, int OMODE, bool SQ>
-__device__ __noinline__ double chunk_c(double* in, double* __restrict__ gdst, int L0, int nlines) {
+// fma sequence as lines_chunk).  The operator reads are constant-bank loads that ptxas
+// turns into LDCUs into uniform registers feeding the DFMAs.  __noinline__: inlined into
+// the group loop, ptxas hoisted all P1^2 operator values out of the loop into regular
+// registers (255 registers + spills at P1 = 13); as a call, each chunk re-reads them.
+// Inside the call n is warp-uniform, so with the n loop rolled (BC_CST_NUNROLL) the reads
+// are LDCUs with a uniform-register index (~1 KB of code per stage instead of ~16 KB
+// fully unrolled: the unrolled stages missed the instruction cache, 17% of stalls).
+// Output modes (k = output index along AXIS, line offset base):
+//   OUT_SMEM        dst[base + k*STRIDE] = y           (dst == in: in place; every read of a
+//                   line precedes its writes, and a line belongs to one lane)
+//   OUT_SMEM_ADD    dst[base + k*STRIDE] = add[base + k*STRIDE] + y
+//   OUT_GLOBAL      gdst[gofs(L, k)] = y               (streaming; SQ: returns sum y^2)
+//   OUT_GLOBAL_ADD  gdst[gofs(L, k)] = add[base + k*STRIDE] + y
+// TRANS: the operator is applied transposed, M[k][n] = cop[n*P1 + k] (local_grad3_t, ax_e).
+enum { OUT_SMEM = 0, OUT_GLOBAL = 1, OUT_SMEM_ADD = 2, OUT_GLOBAL_ADD = 3 };
+template <int P1, int NA, int AXIS, int RR, int CS, int OPI, int OMODE, bool SQ, bool TRANS>
+__device__ __noinline__ double chunk_c(const double* in, double* dst, const double* add, double* __restrict__ gdst,
+                                       int L0, int nlines) {
     using LN = Line<P1, NA, AXIS, double>;
     int base[RR];
 #pragma unroll
@@ -524,10 +533,7 @@ __device__ __noinline__ double chunk_c(double* in, double* __restrict__ gdst, in
     for (int k = 0; k < P1; ++k)
 #pragma unroll
         for (int r = 0; r < RR; ++r) acc[k][r] = 0.0;
-    // x(L, n+1) is loaded while step n's FMAs run; the n loop stays rolled (BC_CST_NUNROLL):
-    // inside this non-inlined call n is warp-uniform, so the operator reads are LDCUs with
-    // a uniform-register index (code size ~1 KB per stage instead of ~16 KB fully unrolled:
-    // the unrolled stages missed the instruction cache, 17% of stall samples)
+    // x(L, n+1) is loaded while step n's FMAs run
     double x[RR];
 #pragma unroll
     for (int r = 0; r < RR; ++r) x[r] = in[base[r]];
@@ -540,7 +546,7 @@ __device__ __noinline__ double chunk_c(double* in, double* __restrict__ gdst, in
         for (int r = 0; r < RR; ++r) xn[r] = in[base[r] + nn * LN::STRIDE];
 #pragma unroll
         for (int k = 0; k < P1; ++k) {
-            const double o = c_ops[CS][OPI][k * P1 + n];
+            const double o = TRANS ? c_ops[CS][OPI][n * P1 + k] : c_ops[CS][OPI][k * P1 + n];
 #pragma unroll
             for (int r = 0; r < RR; ++r) acc[k][r] = fma(o, x[r], acc[k][r]);
         }
@@ -555,11 +561,15 @@ __device__ __noinline__ double chunk_c(double* in, double* __restrict__ gdst, in
         if (L0 + r * 32 < nlines) {
 #pragma unroll
             for (int k = 0; k < P1; ++k) {
-                if constexpr (OMODE == 0) {
-                    in[base[r] + k * LN::STRIDE] = acc[k][r];
+                const int so = base[r] + k * LN::STRIDE;
+                if constexpr (OMODE == OUT_SMEM) {
+                    dst[so] = acc[k][r];
+                } else if constexpr (OMODE == OUT_SMEM_ADD) {
+                    dst[so] = add[so] + acc[k][r];
                 } else {
-                    st_cs(gdst + LN::gofs(L0 + r * 32, k), acc[k][r]);
-                    if constexpr (SQ) sq[r] = fma(acc[k][r], acc[k][r], sq[r]);
+                    const double v = (OMODE == OUT_GLOBAL_ADD) ? add[so] + acc[k][r] : acc[k][r];
+                    st_cs(gdst + LN::gofs(L0 + r * 32, k), v);
+                    if constexpr (SQ) sq[r] = fma(v, v, sq[r]);
                 }
             }
         }
@@ -571,22 +581,24 @@ __device__ __noinline__ double chunk_c(double* in, double* __restrict__ gdst, in
 }
 
 // apply_lines with operator OPI of constant slot CS (same warp-chunked line assignment as
-// apply_lines_w); returns this thread's sum of squares of its outputs (SQ) or 0.
-template <int P1, int NA, int AXIS, int R, int NT, int CS, int OPI, int OMODE, bool SQ = false>
-__device__ __forceinline__ double apply_lines_c(double* in, double* gdst, int nlines) {
+// apply_lines_w): reads `in`, writes per OMODE; returns this thread's sum of squares of
+// its outputs (SQ) or 0.
+template <int P1, int NA, int AXIS, int R, int NT, int CS, int OPI, int OMODE, bool SQ = false, bool TRANS = false>
+__device__ __forceinline__ double apply_lines_c(const double* in, double* dst, const double* add, double* gdst,
+                                                int nlines) {
     constexpr int NW = NT / 32, CH = 32 * R;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int nfull = nlines / CH;
     double sq = 0.0;
     for (int c = warp; c < nfull; c += NW)
-        sq += chunk_c<P1, NA, AXIS, R, CS, OPI, OMODE, SQ>(in, gdst, c * CH + lane, nlines);
+        sq += chunk_c<P1, NA, AXIS, R, CS, OPI, OMODE, SQ, TRANS>(in, dst, add, gdst, c * CH + lane, nlines);
     const int rest = nlines - nfull * CH;
     if (rest > 0 && warp == nfull % NW) {
         const int L0 = nfull * CH + lane, rr = (rest + 31) >> 5;
-        if constexpr (R >= 4) if (rr == 4) return sq + chunk_c<P1, NA, AXIS, 4, CS, OPI, OMODE, SQ>(in, gdst, L0, nlines);
-        if constexpr (R >= 3) if (rr == 3) return sq + chunk_c<P1, NA, AXIS, (R >= 3 ? 3 : 1), CS, OPI, OMODE, SQ>(in, gdst, L0, nlines);
-        if constexpr (R >= 2) if (rr == 2) return sq + chunk_c<P1, NA, AXIS, (R >= 2 ? 2 : 1), CS, OPI, OMODE, SQ>(in, gdst, L0, nlines);
-        sq += chunk_c<P1, NA, AXIS, 1, CS, OPI, OMODE, SQ>(in, gdst, L0, nlines);
+        if constexpr (R >= 4) if (rr == 4) return sq + chunk_c<P1, NA, AXIS, 4, CS, OPI, OMODE, SQ, TRANS>(in, dst, add, gdst, L0, nlines);
+        if constexpr (R >= 3) if (rr == 3) return sq + chunk_c<P1, NA, AXIS, (R >= 3 ? 3 : 1), CS, OPI, OMODE, SQ, TRANS>(in, dst, add, gdst, L0, nlines);
+        if constexpr (R >= 2) if (rr == 2) return sq + chunk_c<P1, NA, AXIS, (R >= 2 ? 2 : 1), CS, OPI, OMODE, SQ, TRANS>(in, dst, add, gdst, L0, nlines);
+        sq += chunk_c<P1, NA, AXIS, 1, CS, OPI, OMODE, SQ, TRANS>(in, dst, add, gdst, L0, nlines);
     }
     return sq;
 }
@@ -629,11 +641,11 @@ sumfact3d_kernel(int64_t N, const T* __restrict__ A, const T* __restrict__ B, co
         };
         if constexpr (CST) {
             constexpr int C = CST ? CS : 0;
-            apply_lines_c<P1, P1, 2, R, NT, C, 0, 0>(in, nullptr, nlines);
+            apply_lines_c<P1, P1, 2, R, NT, C, 0, OUT_SMEM>(in, in, nullptr, nullptr, nlines);
             __syncthreads();
-            apply_lines_c<P1, P1, 1, R, NT, C, 1, 0>(in, nullptr, nlines);
+            apply_lines_c<P1, P1, 1, R, NT, C, 1, OUT_SMEM>(in, in, nullptr, nullptr, nlines);
             __syncthreads();
-            sq += apply_lines_c<P1, P1, 0, R, NT, C, 2, 1, true>(in, Vg, nlines);
+            sq += apply_lines_c<P1, P1, 0, R, NT, C, 2, OUT_GLOBAL, true>(in, nullptr, nullptr, Vg, nlines);
         } else {
             apply_lines<P1, P1, 2, R, NT>(in, opA, nlines, s1);
             __syncthreads();
@@ -702,9 +714,9 @@ sumfact2d_kernel(int64_t N, const double* __restrict__ A, const double* __restri
         auto st2 = [&](int L, int, int k, T v) { st_cs(Vg + Line<P1, 1, 1, T>::gofs(L, k), v); };
         if constexpr (CST) {
             constexpr int C = CST ? CS : 0;
-            apply_lines_c<P1, 1, 2, R, NT, C, 0, 0>(in, nullptr, nlines);
+            apply_lines_c<P1, 1, 2, R, NT, C, 0, OUT_SMEM>(in, in, nullptr, nullptr, nlines);
             __syncthreads();
-            apply_lines_c<P1, 1, 1, R, NT, C, 1, 1>(in, Vg, nlines);
+            apply_lines_c<P1, 1, 1, R, NT, C, 1, OUT_GLOBAL>(in, nullptr, nullptr, Vg, nlines);
         } else {
             apply_lines<P1, 1, 2, R, NT, T, decltype(st1), U>(in, opA, nlines, st1);
             __syncthreads();
@@ -760,10 +772,10 @@ local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __rest
         const int64_t gbase = e0 * G::NPTS;
         if constexpr (CST) {
             constexpr int C = CST ? CS : 0;
-            apply_lines_c<P1, P1, 1, R, NT, C, 0, 1>(in, us + gbase, nlines);
-            apply_lines_c<P1, P1, 0, R, NT, C, 0, 1>(in, ut + gbase, nlines);
+            apply_lines_c<P1, P1, 1, R, NT, C, 0, OUT_GLOBAL>(in, nullptr, nullptr, us + gbase, nlines);
+            apply_lines_c<P1, P1, 0, R, NT, C, 0, OUT_GLOBAL>(in, nullptr, nullptr, ut + gbase, nlines);
             __syncthreads();
-            apply_lines_c<P1, P1, 2, R, NT, C, 0, 0>(in, nullptr, nlines);
+            apply_lines_c<P1, P1, 2, R, NT, C, 0, OUT_SMEM>(in, in, nullptr, nullptr, nlines);
         } else {
             apply_lines<P1, P1, 1, R, NT>(in, opD, nlines, [&](int L, int, int k, T v) {
                 st_cs(us + gbase + Line<P1, P1, 1, T>::gofs(L, k), v);
@@ -809,12 +821,14 @@ int launch_local_grad3(int64_t N, const double* D, const double* U, double* ur, 
 // ====================================================================== local_grad3_t
 //   U = D^T along axis 2 of ur + D^T along axis 1 of us + D^T along axis 0 of ut,
 //   partial sums added in the order (r + s) + t.  Three field buffers, all in place.
-template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, 3, K_LG3T>::NT)
+template <int P1, int CS>
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 3, K_LG3T, (CS >= 0)>::NT)
 local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ ur,
                      const double* __restrict__ us, const double* __restrict__ ut, double* __restrict__ U) {
     using T = double;
-    using CF = Cfg<P1, P1, T, 3, K_LG3T>;
+    constexpr bool CST = CS >= 0;
+    constexpr int C = CST ? CS : 0;
+    using CF = Cfg<P1, P1, T, 3, K_LG3T, CST>;
     using G = Geo<P1, P1, T>;
     constexpr int E = CF::E, NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -822,7 +836,7 @@ local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __re
     T* bR0 = opT + 2 * op_elems<P1, T>();
     T* bS0 = bR0 + CF::BUF;
     T* bT0 = bS0 + CF::BUF;
-    load_op<P1, T, NT, true>(opT, D);
+    if constexpr (!CST) load_op<P1, T, NT, true>(opT, D);
     const int64_t ngroups = (N + E - 1) / E;
     for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
         const int64_t e0 = g * E;
@@ -840,41 +854,66 @@ local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __re
         cp_async_commit();
         cp_async_wait_n<2>();
         __syncthreads();
-        apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
+        if constexpr (CST)
+            apply_lines_c<P1, P1, 2, R, NT, C, 0, OUT_SMEM, false, true>(bR, bR, nullptr, nullptr, nlines);
+        else
+            apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
         cp_async_wait_n<1>();
         __syncthreads();
-        apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines, [&](int, int base, int k, T v) {
-            bS[base + k * G::RS] = bR[base + k * G::RS] + v;
-        });
+        if constexpr (CST)
+            apply_lines_c<P1, P1, 1, R, NT, C, 0, OUT_SMEM_ADD, false, true>(bS, bS, bR, nullptr, nlines);
+        else
+            apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines, [&](int, int base, int k, T v) {
+                bS[base + k * G::RS] = bR[base + k * G::RS] + v;
+            });
         cp_async_wait_n<0>();
         __syncthreads();
-        apply_lines<P1, P1, 0, R, NT>(bT, opT, nlines, [&](int L, int base, int k, T v) {
-            st_cs(U + gbase + Line<P1, P1, 0, T>::gofs(L, k), bS[base + k * G::PS] + v);
-        });
+        if constexpr (CST)
+            apply_lines_c<P1, P1, 0, R, NT, C, 0, OUT_GLOBAL_ADD, false, true>(bT, nullptr, bS, U + gbase, nlines);
+        else
+            apply_lines<P1, P1, 0, R, NT>(bT, opT, nlines, [&](int L, int base, int k, T v) {
+                st_cs(U + gbase + Line<P1, P1, 0, T>::gofs(L, k), bS[base + k * G::PS] + v);
+            });
     }
+}
+
+template <int P1, int CS>
+int launch_local_grad3_t_k(int64_t N, const double* D, const double* ur, const double* us, const double* ut,
+                           double* U, cudaStream_t s) {
+    using CF = Cfg<P1, P1, double, 3, K_LG3T, (CS >= 0)>;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
+    const int64_t ngroups = (N + CF::E - 1) / CF::E;
+    const int grid = grid_for(local_grad3_t_kernel<P1, CS>, CF::NT, CF::SMEM, ngroups, &occ);
+    local_grad3_t_kernel<P1, CS><<<grid, CF::NT, CF::SMEM, s>>>(N, D, ur, us, ut, U);
+    const int st = launch_status();
+    if (CS >= 0) op_slot_release(s, CS);
+    return st;
 }
 
 template <int P1>
 int launch_local_grad3_t(int64_t N, const double* D, const double* ur, const double* us, const double* ut,
                          double* U, cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, 3, K_LG3T>;
-    static PerDevice<int> occ_dev;
-    int& occ = occ_dev.get();
-    const int64_t ngroups = (N + CF::E - 1) / CF::E;
-    const int grid = grid_for(local_grad3_t_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
-    local_grad3_t_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, D, ur, us, ut, U);
-    return launch_status();
+    if (N >= OPS_CONST_MIN_N) {
+        int slot, st;
+        if ((st = op_slot_acquire(s, &D, 1, P1, &slot))) return st;
+        return slot == 0 ? launch_local_grad3_t_k<P1, 0>(N, D, ur, us, ut, U, s)
+                         : launch_local_grad3_t_k<P1, 1>(N, D, ur, us, ut, U, s);
+    }
+    return launch_local_grad3_t_k<P1, -1>(N, D, ur, us, ut, U, s);
 }
 
 // ====================================================================== ax_e
 // (us, ut) from U into two buffers; ur in place over U; per-point geometric mixing in
 // place; then local_grad3_t in place as above.  Three field buffers.
-template <int P1>
-__global__ void __launch_bounds__(Cfg<P1, P1, double, 3, K_AXE>::NT)
+template <int P1, int CS>
+__global__ void __launch_bounds__(Cfg<P1, P1, double, 3, K_AXE, (CS >= 0)>::NT)
 ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ Uin,
             const double* __restrict__ Gm, double* __restrict__ Wout) {
     using T = double;
-    using CF = Cfg<P1, P1, T, 3, K_AXE>;
+    constexpr bool CST = CS >= 0;
+    constexpr int C = CST ? CS : 0;
+    using CF = Cfg<P1, P1, T, 3, K_AXE, CST>;
     using G = Geo<P1, P1, T>;
     constexpr int E = CF::E, NT = CF::NT, R = CF::R;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -883,8 +922,10 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
     T* bR0 = opT + op_elems<P1, T>();  // holds U, then ur / wr
     T* bS = bR0 + CF::BUF;
     T* bT = bS + CF::BUF;
-    load_op<P1, T, NT>(opD, D);
-    load_op<P1, T, NT, true>(opT, D);
+    if constexpr (!CST) {
+        load_op<P1, T, NT>(opD, D);
+        load_op<P1, T, NT, true>(opT, D);
+    }
     const int64_t ngroups = (N + E - 1) / E;
     for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
         const int64_t e0 = g * E;
@@ -896,10 +937,17 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
         cp_async_commit();
         cp_async_wait_all();
         __syncthreads();
-        apply_lines<P1, P1, 1, R, NT>(bR, opD, nlines, [&](int, int base, int k, T v) { bS[base + k * G::RS] = v; });
-        apply_lines<P1, P1, 0, R, NT>(bR, opD, nlines, [&](int, int base, int k, T v) { bT[base + k * G::PS] = v; });
-        __syncthreads();
-        apply_lines<P1, P1, 2, R, NT>(bR, opD, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
+        if constexpr (CST) {
+            apply_lines_c<P1, P1, 1, R, NT, C, 0, OUT_SMEM>(bR, bS, nullptr, nullptr, nlines);
+            apply_lines_c<P1, P1, 0, R, NT, C, 0, OUT_SMEM>(bR, bT, nullptr, nullptr, nlines);
+            __syncthreads();
+            apply_lines_c<P1, P1, 2, R, NT, C, 0, OUT_SMEM>(bR, bR, nullptr, nullptr, nlines);
+        } else {
+            apply_lines<P1, P1, 1, R, NT>(bR, opD, nlines, [&](int, int base, int k, T v) { bS[base + k * G::RS] = v; });
+            apply_lines<P1, P1, 0, R, NT>(bR, opD, nlines, [&](int, int base, int k, T v) { bT[base + k * G::PS] = v; });
+            __syncthreads();
+            apply_lines<P1, P1, 2, R, NT>(bR, opD, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
+        }
         __syncthreads();
         const int total = ne * G::NPTS;
         // G[e][c][q]: AXE_PB points per thread per batch, all 6*AXE_PB loads issued before use
@@ -928,27 +976,47 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
             }
         }
         __syncthreads();
-        apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
-        __syncthreads();
-        apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines, [&](int, int base, int k, T v) {
-            bS[base + k * G::RS] = bR[base + k * G::RS] + v;
-        });
-        __syncthreads();
-        apply_lines<P1, P1, 0, R, NT>(bT, opT, nlines, [&](int L, int base, int k, T v) {
-            st_cs(Wout + gbase + Line<P1, P1, 0, T>::gofs(L, k), bS[base + k * G::PS] + v);
-        });
+        if constexpr (CST) {
+            apply_lines_c<P1, P1, 2, R, NT, C, 0, OUT_SMEM, false, true>(bR, bR, nullptr, nullptr, nlines);
+            __syncthreads();
+            apply_lines_c<P1, P1, 1, R, NT, C, 0, OUT_SMEM_ADD, false, true>(bS, bS, bR, nullptr, nlines);
+            __syncthreads();
+            apply_lines_c<P1, P1, 0, R, NT, C, 0, OUT_GLOBAL_ADD, false, true>(bT, nullptr, bS, Wout + gbase, nlines);
+        } else {
+            apply_lines<P1, P1, 2, R, NT>(bR, opT, nlines, [&](int, int base, int k, T v) { bR[base + k] = v; });
+            __syncthreads();
+            apply_lines<P1, P1, 1, R, NT>(bS, opT, nlines, [&](int, int base, int k, T v) {
+                bS[base + k * G::RS] = bR[base + k * G::RS] + v;
+            });
+            __syncthreads();
+            apply_lines<P1, P1, 0, R, NT>(bT, opT, nlines, [&](int L, int base, int k, T v) {
+                st_cs(Wout + gbase + Line<P1, P1, 0, T>::gofs(L, k), bS[base + k * G::PS] + v);
+            });
+        }
     }
+}
+
+template <int P1, int CS>
+int launch_ax_e_k(int64_t N, const double* D, const double* U, const double* Gm, double* W, cudaStream_t s) {
+    using CF = Cfg<P1, P1, double, 3, K_AXE, (CS >= 0)>;
+    static PerDevice<int> occ_dev;
+    int& occ = occ_dev.get();
+    const int64_t ngroups = (N + CF::E - 1) / CF::E;
+    const int grid = grid_for(ax_e_kernel<P1, CS>, CF::NT, CF::SMEM, ngroups, &occ);
+    ax_e_kernel<P1, CS><<<grid, CF::NT, CF::SMEM, s>>>(N, D, U, Gm, W);
+    const int st = launch_status();
+    if (CS >= 0) op_slot_release(s, CS);
+    return st;
 }
 
 template <int P1>
 int launch_ax_e(int64_t N, const double* D, const double* U, const double* Gm, double* W, cudaStream_t s) {
-    using CF = Cfg<P1, P1, double, 3, K_AXE>;
-    static PerDevice<int> occ_dev;
-    int& occ = occ_dev.get();
-    const int64_t ngroups = (N + CF::E - 1) / CF::E;
-    const int grid = grid_for(ax_e_kernel<P1>, CF::NT, CF::SMEM, ngroups, &occ);
-    ax_e_kernel<P1><<<grid, CF::NT, CF::SMEM, s>>>(N, D, U, Gm, W);
-    return launch_status();
+    if (N >= OPS_CONST_MIN_N) {
+        int slot, st;
+        if ((st = op_slot_acquire(s, &D, 1, P1, &slot))) return st;
+        return slot == 0 ? launch_ax_e_k<P1, 0>(N, D, U, Gm, W, s) : launch_ax_e_k<P1, 1>(N, D, U, Gm, W, s);
+    }
+    return launch_ax_e_k<P1, -1>(N, D, U, Gm, W, s);
 }
 
 // ---------------------------------------------------------------- constant-bank slots (host)

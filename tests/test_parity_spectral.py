@@ -102,16 +102,16 @@ def test_local_grad3(bc, P1):
 @pytest.mark.parametrize("P1", ALL_P1)
 def test_local_grad3_t(bc, P1):
     D = syn.tensor(6, (P1, P1), kind=syn.KIND_INT)
-    N = 11
-    ur, us, ut = (syn.tensor(t, (N, P1, P1, P1), kind=syn.KIND_INT) for t in (7, 8, 9))
-    got = bc.local_grad3_t(to_dev(D), to_dev(ur), to_dev(us), to_dev(ut), out=poisoned_like(to_dev(ur)))
-    assert np.array_equal(to_host(got), oracle.local_grad3_t(D, ur, us, ut))
+    for N in (11, 150):  # shared-memory and constant-bank operator kernels
+        ur, us, ut = (syn.tensor(t, (N, P1, P1, P1), kind=syn.KIND_INT) for t in (7, 8, 9))
+        got = bc.local_grad3_t(to_dev(D), to_dev(ur), to_dev(us), to_dev(ut), out=poisoned_like(to_dev(ur)))
+        assert np.array_equal(to_host(got), oracle.local_grad3_t(D, ur, us, ut)), f"P1={P1} N={N}"
 
 
+@pytest.mark.parametrize("N", [7, 140])
 @pytest.mark.parametrize("P1", [2, 5, 8, 12, 13, 16])
-def test_ax_e(bc, P1):
+def test_ax_e(bc, P1, N):
     D = syn.gll_derivative(P1 - 1)
-    N = 7
     U = syn.tensor(1, (N, P1, P1, P1))
     G = syn.tensor(11, (N, 6, P1, P1, P1))
     got = bc.ax_e(to_dev(D), to_dev(U), to_dev(G), out=poisoned_like(to_dev(U)))
