@@ -368,8 +368,14 @@ enum SpecKernel { K_SF3 = 0, K_SF2 = 1, K_LG3 = 2, K_LG3T = 3, K_AXE = 4 };
 #ifndef BC_CST_R
 #define BC_CST_R 0  // lines per thread of the constant-bank-operator kernels (0: as the smem ones)
 #endif
+#ifndef BC_CST_R_SF3
+#define BC_CST_R_SF3 0  // sumfact3d lines per thread with constant-bank operators (0: table)
+#endif
 #ifndef BC_CST_NUNROLL
 #define BC_CST_NUNROLL 2  // unroll of the constant-operator stages' n loop (measured: 2 >= 1)
+#endif
+#ifndef BC_CST_PF_SF3
+#define BC_CST_PF_SF3 0  // sumfact3d with constant-bank operators: prefetch the next group
 #endif
 #ifndef BC_CST_PF
 #define BC_CST_PF -1  // constant-bank-operator kernels: -1 = prefetch as the smem table, 0/1 = off/on
@@ -397,9 +403,10 @@ struct SpecTable {
     // 128 threads x R = 4 (1% idle lanes instead of 12% with E = 2 on 96 threads)
     static constexpr int EF = (SF3LG3 && P1 == 13) ? BC_E13 : ((KIND == K_SF2 && P1 == 13) ? BC_E13_SF2 : 0);
     // lines per thread with constant-bank operators (tools/sweep_spectral.py, DESIGN.md
-    // §4.1): 4, except sumfact2d at P1 >= 12 (2)
+    // §4.1): 4, except sumfact2d at P1 >= 12 (3) and the 3-field kernels (2)
     static constexpr int RC = BC_CST_R ? BC_CST_R
-                                       : ((KIND == K_SF2 && P1 >= 12) || KIND == K_LG3T || KIND == K_AXE ? 2 : 4);
+                                       : ((KIND == K_SF3 && BC_CST_R_SF3) ? BC_CST_R_SF3
+                                       : (KIND == K_SF2 && P1 >= 12) ? 3 : (KIND == K_LG3T || KIND == K_AXE ? 2 : 4));
     // unroll of the contracted-index loop: sumfact2d fully (its two stages fit the registers)
     static constexpr int UNROLL = (KIND == K_SF2 && BC_SF2_UNROLL && P1 >= 9) ? P1 : BC_NUNROLL;
 };
@@ -408,14 +415,19 @@ template <int P1, int NA, typename T, int NBUF_FIELDS, int KIND = K_SF3, bool CS
 struct Cfg {
     using G = Geo<P1, NA, T>;
     using TB = SpecTable<P1, KIND>;
-    static constexpr bool PREFETCH = ((CST && BC_CST_PF >= 0) ? (bool)BC_CST_PF : TB::PREFETCH) &&
+    static constexpr bool PREFETCH = ((CST && KIND == K_SF3 && BC_CST_PF_SF3) ? true
+                                      : ((CST && BC_CST_PF >= 0) ? (bool)BC_CST_PF : TB::PREFETCH)) &&
                                      NBUF_FIELDS == 1;  // single-field kernels only
     static constexpr int NBUF = NBUF_FIELDS + (PREFETCH ? 1 : 0);
     static constexpr int BUF_BYTES = TB::BUF_KB * 1024;  // target bytes per element-group buffer
     static constexpr int E0 = BUF_BYTES / (G::ES * (int)sizeof(T));
     // even by default; a measured table entry may force E (odd E x odd P1 groups start 8 bytes
     // off a 16-byte boundary, handled by load_group_async)
-    static constexpr int E = (CST && BC_CST_E && P1 >= 10) ? BC_CST_E : (TB::EF ? TB::EF : (E0 < 2 ? 1 : (E0 & ~1)));
+    // (measured with constant-bank operators: local_grad3 at P1 = 13 with 4-element groups,
+    // 0.805 -> 0.822 of HBM; sumfact3d keeps 3)
+    static constexpr int E = (CST && BC_CST_E && P1 >= 10) ? BC_CST_E
+                           : (CST && KIND == K_LG3 && P1 == 13) ? 4
+                           : (TB::EF ? TB::EF : (E0 < 2 ? 1 : (E0 & ~1)));
     static constexpr int R = CST ? TB::RC : TB::R;
     static constexpr int LINES = E * NA * P1;  // lines per axis per group (E * NPTS / P1)
     static constexpr int NT0 = ((LINES + R - 1) / R + 31) / 32 * 32;
