@@ -124,6 +124,21 @@ class ClockSampler:
                 "samples": len(sm), "gpu": self.index}
 
 
+def gather_clocks(local, rank):
+    """Every rank samples its own GPU; rank 0 reports the median over ranks' medians, the
+    lowest max clock, the union of throttle reasons and the per-rank summaries."""
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size() == 1:
+        return local
+    allc = [None] * dist.get_world_size()
+    dist.all_gather_object(allc, local)
+    sm = [c["sm_mhz"] for c in allc if c.get("sm_mhz") is not None]
+    mx = [c["sm_max_mhz"] for c in allc if c.get("sm_max_mhz") is not None]
+    reasons = sorted({r for c in allc for r in c.get("reasons", [])})
+    return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": min(mx) if mx else None,
+            "reasons": reasons, "samples": sum(c.get("samples", 0) for c in allc), "per_rank": allc}
+
+
 def env_rank():
     return int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1"))
 
@@ -550,7 +565,7 @@ def main():
             e2e = measure_e2e(args, step, rank, dev, stream, flops_all, step.checks.cpu().clone())
         except (RuntimeError, MemoryError) as exc:  # e.g. pinned host memory exhausted with many ranks
             e2e = {"value": None, "unit": "GFLOP/s", "error": f"{type(exc).__name__}: {str(exc)[:160]}"}
-    clk = clocks.summary()
+    clk = gather_clocks(clocks.summary(), rank)
     del step
     torch.cuda.empty_cache()
 
