@@ -380,46 +380,12 @@ struct TmaGeo {
     static constexpr size_t SMEM = 1024 + (size_t)NS * STAGE_BYTES + ACC * 8 + 2 * NS * 8;
 };
 
-__device__ __forceinline__ void mbar_init(uint32_t bar, int count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(bar), "r"(count));
-}
-__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, int bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(bar) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint32_t bar, int parity) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n"
-        "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-        "@!p bra WAIT_%=;\n}\n" ::"r"(bar), "r"(parity) : "memory");
-}
 __device__ __forceinline__ void tma_load_4d(uint32_t dst, const CUtensorMap* map, int c0, int c1, int c2, int c3,
                                             uint32_t bar) {
     asm volatile(
         "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], [%6];\n"
         ::"r"(dst), "l"(map), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(bar) : "memory");
 }
-__device__ __forceinline__ void named_bar_sync(int id, int n) {
-    asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(n) : "memory");
-}
-
-// Consumer warp releases a ring slot it has finished reading.  The slot's next contents
-// are written by TMA, i.e. by the ASYNC proxy, while the consumers read it with ordinary
-// ld.shared (the GENERIC proxy); the mbarrier release/acquire pair orders the two only
-// after a proxy fence: without `fence.proxy.async`, ptxas issues the arrive while the
-// stage's last ld.shared are still in flight and the producer's refill can overwrite a
-// fragment before it is read (measured: 183 of 200 repeat runs of the tile-16 fused
-// kernel corrupted 128-1648 t3 values, one warp m-tile each; with the fence 0 of 200 —
-// DESIGN.md §4.2).  Every lane fences its own reads, then lane 0 arrives for the warp.
-__device__ __forceinline__ void release_slot(uint32_t bar_empty_slot, int lane) {
-    asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-    __syncwarp();
-    if (lane == 0) mbar_arrive(bar_empty_slot);
-}
-
 // fragment loads as volatile asm: kept in program order relative to the (volatile) DMMAs,
 // so a stage's fragments are all loaded into distinct registers before its first DMMA
 // (plain loads let ptxas reuse one register per fragment and expose the LDS latency

@@ -12,6 +12,7 @@
 // (fusion); only U in and the outputs touch HBM.
 #include <algorithm>
 #include <mutex>
+#include <type_traits>
 
 #include "common.cuh"
 
@@ -530,7 +531,7 @@ void op_slot_release(cudaStream_t s, int slot);
 //   OUT_GLOBAL_ADD  gdst[gofs(L, k)] = add[base + k*STRIDE] + y
 // TRANS: the operator is applied transposed, M[k][n] = cop[n*P1 + k] (local_grad3_t, ax_e).
 enum { OUT_SMEM = 0, OUT_GLOBAL = 1, OUT_SMEM_ADD = 2, OUT_GLOBAL_ADD = 3 };
-template <int P1, int NA, int AXIS, int RR, int CS, int OPI, int OMODE, bool SQ, bool TRANS>
+template <int P1, int NA, int AXIS, int RR, int CS, int OPI, int OMODE, bool SQ, bool TRANS, int NUNR = BC_CST_NUNROLL>
 __device__ __noinline__ double chunk_c(const double* in, double* dst, const double* add, double* __restrict__ gdst,
                                        int L0, int nlines) {
     using LN = Line<P1, NA, AXIS, double>;
@@ -549,7 +550,6 @@ __device__ __noinline__ double chunk_c(const double* in, double* dst, const doub
     double x[RR];
 #pragma unroll
     for (int r = 0; r < RR; ++r) x[r] = in[base[r]];
-    constexpr int NUNR = BC_CST_NUNROLL;
 #pragma unroll NUNR
     for (int n = 0; n < P1; ++n) {
         double xn[RR];
@@ -595,24 +595,34 @@ __device__ __noinline__ double chunk_c(const double* in, double* dst, const doub
 // apply_lines with operator OPI of constant slot CS (same warp-chunked line assignment as
 // apply_lines_w): reads `in`, writes per OMODE; returns this thread's sum of squares of
 // its outputs (SQ) or 0.
-template <int P1, int NA, int AXIS, int R, int NT, int CS, int OPI, int OMODE, bool SQ = false, bool TRANS = false>
-__device__ __forceinline__ double apply_lines_c(const double* in, double* dst, const double* add, double* gdst,
-                                                int nlines) {
-    constexpr int NW = NT / 32, CH = 32 * R;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+// apply_lines_gc: the same over NW warps of which this is warp `warp` (a consumer group of
+// a warp-specialised kernel); apply_lines_c: all NT threads of the CTA.
+template <int P1, int NA, int AXIS, int R, int NW, int CS, int OPI, int OMODE, bool SQ = false, bool TRANS = false,
+          int NUNR = BC_CST_NUNROLL>
+__device__ __forceinline__ double apply_lines_gc(int warp, const double* in, double* dst, const double* add,
+                                                 double* gdst, int nlines) {
+    constexpr int CH = 32 * R;
+    const int lane = threadIdx.x & 31;
     const int nfull = nlines / CH;
     double sq = 0.0;
     for (int c = warp; c < nfull; c += NW)
-        sq += chunk_c<P1, NA, AXIS, R, CS, OPI, OMODE, SQ, TRANS>(in, dst, add, gdst, c * CH + lane, nlines);
+        sq += chunk_c<P1, NA, AXIS, R, CS, OPI, OMODE, SQ, TRANS, NUNR>(in, dst, add, gdst, c * CH + lane, nlines);
     const int rest = nlines - nfull * CH;
     if (rest > 0 && warp == nfull % NW) {
         const int L0 = nfull * CH + lane, rr = (rest + 31) >> 5;
-        if constexpr (R >= 4) if (rr == 4) return sq + chunk_c<P1, NA, AXIS, 4, CS, OPI, OMODE, SQ, TRANS>(in, dst, add, gdst, L0, nlines);
-        if constexpr (R >= 3) if (rr == 3) return sq + chunk_c<P1, NA, AXIS, (R >= 3 ? 3 : 1), CS, OPI, OMODE, SQ, TRANS>(in, dst, add, gdst, L0, nlines);
-        if constexpr (R >= 2) if (rr == 2) return sq + chunk_c<P1, NA, AXIS, (R >= 2 ? 2 : 1), CS, OPI, OMODE, SQ, TRANS>(in, dst, add, gdst, L0, nlines);
-        sq += chunk_c<P1, NA, AXIS, 1, CS, OPI, OMODE, SQ, TRANS>(in, dst, add, gdst, L0, nlines);
+        if constexpr (R >= 4) if (rr == 4) return sq + chunk_c<P1, NA, AXIS, 4, CS, OPI, OMODE, SQ, TRANS, NUNR>(in, dst, add, gdst, L0, nlines);
+        if constexpr (R >= 3) if (rr == 3) return sq + chunk_c<P1, NA, AXIS, (R >= 3 ? 3 : 1), CS, OPI, OMODE, SQ, TRANS, NUNR>(in, dst, add, gdst, L0, nlines);
+        if constexpr (R >= 2) if (rr == 2) return sq + chunk_c<P1, NA, AXIS, (R >= 2 ? 2 : 1), CS, OPI, OMODE, SQ, TRANS, NUNR>(in, dst, add, gdst, L0, nlines);
+        sq += chunk_c<P1, NA, AXIS, 1, CS, OPI, OMODE, SQ, TRANS, NUNR>(in, dst, add, gdst, L0, nlines);
     }
     return sq;
+}
+
+template <int P1, int NA, int AXIS, int R, int NT, int CS, int OPI, int OMODE, bool SQ = false, bool TRANS = false>
+__device__ __forceinline__ double apply_lines_c(const double* in, double* dst, const double* add, double* gdst,
+                                                int nlines) {
+    return apply_lines_gc<P1, NA, AXIS, R, NT / 32, CS, OPI, OMODE, SQ, TRANS>(threadIdx.x >> 5, in, dst, add, gdst,
+                                                                               nlines);
 }
 
 // ====================================================================== sumfact3d
@@ -685,6 +695,210 @@ int launch_sumfact3d_k(int64_t N, const T* A, const T* B, const T* C, const T* U
     return run_check_finalize(grid, ws, s);
 }
 
+// ------------------------------------------------------------ sumfact3d, TMA element ring
+// Warp-specialised persistent form of sumfact3d_kernel for odd P1 (smem layout == global
+// layout, no row padding), constant-bank operators.  One CTA per SM:
+//   * a loader warp streams items (E consecutive elements, E*P1^3*8 bytes, a multiple of 16
+//     for even E) into an NB-slot shared-memory ring with 1-D bulk copies (TMA engine,
+//     cp.async.bulk ... mbarrier::complete_tx), full/empty mbarrier pair per slot;
+//   * NG consumer groups of NWG warps each take items round robin (item j -> group j % NG)
+//     and run S1 -> S2 -> S3 on their slot exactly as sumfact3d_kernel does (S1/S2 in place,
+//     S3 stored from registers, coalesced), separated by the group's named barrier, then
+//     release the slot (generic->async proxy fence, one arrive per warp).
+// The loads of the next NB - NG items are in flight while the groups compute, so no warp
+// waits for its element data (the unbuffered kernel's 18% long-scoreboard stall), and a
+// group's stage barriers stall only that group.
+#ifndef BC_T3_E
+#define BC_T3_E 2
+#endif
+#ifndef BC_T3_NB
+#define BC_T3_NB 5
+#endif
+#ifndef BC_T3_NG
+#define BC_T3_NG 3
+#endif
+#ifndef BC_T3_NWG
+#define BC_T3_NWG 4
+#endif
+#ifndef BC_T3_R
+#define BC_T3_R 3
+#endif
+// Ring geometry: items of E elements of NPTS values, NB slots, NG x NWG consumer warps plus
+// XW service warps (loader; storer).
+template <int NPTS_, int E_, int NB_, int NG_, int NWG_, int R_, int XW>
+struct Ring {
+    static constexpr int E = E_, NB = NB_, NG = NG_, NWG = NWG_, R = R_, NPTS = NPTS_;
+    // doubles per slot: an item may start 8 bytes past a 16-byte boundary (odd E x odd
+    // NPTS); its copy then starts one value early and may end one value late (16-byte
+    // aligned, multiple-of-16 bulk copies), so a slot holds E * NPTS + 2 values
+    static constexpr int SLOT = (E * NPTS + 2 + 1) & ~1;
+    static constexpr int NT = 32 * (NG * NWG + XW);
+    static constexpr size_t SMEM = (size_t)NB * SLOT * 8 + 3 * NB * 8;
+    static constexpr bool FITS = SMEM <= 227 * 1024;
+    static_assert(NB > NG, "ring_wait_full needs more slots than consumer groups");
+};
+// 2-D (sumfact2d) ring: items of E2 elements of P1^2 values (26 x 169 = 2 x 13^3 at P1 = 13)
+#ifndef BC_T2_E
+#define BC_T2_E 0  // 0: as many elements as fill the group's 32 NWG R lanes' lines
+#endif
+#ifndef BC_T2_NB
+#define BC_T2_NB 10
+#endif
+#ifndef BC_T2_NG
+#define BC_T2_NG 6
+#endif
+#ifndef BC_T2_NWG
+#define BC_T2_NWG 2
+#endif
+#ifndef BC_T2_R
+#define BC_T2_R 3
+#endif
+template <int P1, int NA = P1>
+using TmaSf3 = typename std::conditional<
+    NA == 1, Ring<P1 * P1, (BC_T2_E ? BC_T2_E : 32 * BC_T2_NWG * BC_T2_R / P1), BC_T2_NB, BC_T2_NG, BC_T2_NWG, BC_T2_R, 1>,
+    Ring<P1 * P1 * P1, BC_T3_E, BC_T3_NB, BC_T3_NG, BC_T3_NWG, BC_T3_R, 1>>::type;
+
+// item j of this CTA: elements [e0, e0 + ne); its first value sits at slot + item_lead
+__device__ __forceinline__ int item_lead(const double* p) { return (int)((reinterpret_cast<uintptr_t>(p) >> 3) & 1); }
+
+// Loader (one thread): items j = 0 .. nitems-1 of this CTA into slot j % NB.  Copies
+// [src - lead, src - lead + 16 nv) with nv 16-byte units covering the item; where that
+// would read past the field's end (the last item only), the final value is copied by a
+// plain load/store instead, ordered before the consumers' reads by the release of
+// expect_tx.  A slot is refilled after its empty barrier's previous phase completed.
+template <class RG>
+__device__ __forceinline__ void ring_loader(int64_t N, const double* __restrict__ U, double* slots, uint32_t full0,
+                                            uint32_t empty0, int64_t nitems) {
+    for (int64_t j = 0; j < nitems; ++j) {
+        const int b = (int)(j % RG::NB);
+        const int64_t use = j / RG::NB;
+        if (use > 0) mbar_wait(empty0 + 8 * b, (int)((use - 1) & 1));
+        const int64_t e0 = (blockIdx.x + j * gridDim.x) * RG::E;
+        const int ne = (int)imin64(RG::E, N - e0);
+        const double* src = U + e0 * RG::NPTS;
+        const int lead = item_lead(src);
+        const int tot = lead + ne * RG::NPTS;
+        int nv = (tot + 1) >> 1;
+        double* dst = slots + (size_t)b * RG::SLOT;
+        if ((tot & 1) && e0 + ne == N) {
+            nv = tot >> 1;
+            dst[tot - 1] = src[tot - 1 - lead];
+        }
+        mbar_expect_tx(full0 + 8 * b, nv * 16);
+        bulk_load(smem_u32(dst), src - lead, (uint32_t)nv * 16u, full0 + 8 * b);
+    }
+}
+
+// Consumer wait for item j (slot b = j % NB, use u = j / NB).  A parity wait is exact only
+// while the barrier is at most one phase behind the awaited one, and with NG groups sharing
+// the ring a group can reach use u of a slot whose use u-1 (another group's item, its bulk
+// copy still in flight: copies complete out of order) has not completed yet -- the parity
+// of phase u would then read as complete and the group would compute on the previous
+// item's bytes.  So for u >= 1 the consumer first waits for the release of use u-1 (empty
+// phase u-1, which implies full phase u-1 completed), then for full phase u.  The empty
+// wait itself cannot alias: this group consumed item j - NG > j - NB, so the loader had
+// passed its wait for empty phase u-2.  (Found as intermittent 'unspecified launch failure'
+// at large N: the mis-synchronised group's release over-arrived the empty barrier and the
+// ring's transaction accounting broke.)
+template <int NB>
+__device__ __forceinline__ void ring_wait_full(uint32_t full0, uint32_t empty0, int b, int64_t j) {
+    const int64_t use = j / NB;
+    if (use > 0) mbar_wait(empty0 + 8 * b, (int)((use - 1) & 1));
+    mbar_wait(full0 + 8 * b, (int)(use & 1));
+}
+
+// NA = P1: sumfact3d (S1, S2 in place, S3 to V);  NA = 1: sumfact2d (W in place, V = B W).
+template <int P1, int NA, int CS>
+__global__ void __launch_bounds__(TmaSf3<P1, NA>::NT, 1)
+sumfact_tma_kernel(int64_t N, const double* __restrict__ U, double* __restrict__ V, double* __restrict__ ws) {
+    using TC = TmaSf3<P1, NA>;
+    constexpr int E = TC::E, NB = TC::NB, NG = TC::NG, NWG = TC::NWG, NPTS = TC::NPTS;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    double* slots = reinterpret_cast<double*>(smem_raw);
+    const uint32_t full0 = smem_u32(smem_raw + (size_t)NB * TC::SLOT * 8), empty0 = full0 + 8 * NB;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int b = 0; b < NB; ++b) {
+            mbar_init(full0 + 8 * b, 1);
+            mbar_init(empty0 + 8 * b, NWG);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const int64_t ngroups = (N + E - 1) / E;
+    const int64_t nitems = ngroups > blockIdx.x ? (ngroups - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    double sq = 0.0;
+    if (warp == NG * NWG) {
+        if (lane == 0) ring_loader<TC>(N, U, slots, full0, empty0, nitems);
+    } else {
+        constexpr int C = CS;
+        const int grp = warp / NWG, wg = warp - grp * NWG;
+        for (int64_t j = grp; j < nitems; j += NG) {
+            const int b = (int)(j % NB);
+            ring_wait_full<NB>(full0, empty0, b, j);
+            const int64_t e0 = (blockIdx.x + j * gridDim.x) * E;
+            const int nlines = (int)imin64(E, N - e0) * NA * P1;
+            double* in = slots + (size_t)b * TC::SLOT + item_lead(U + e0 * NPTS);
+            apply_lines_gc<P1, NA, 2, TC::R, NWG, C, 0, OUT_SMEM>(wg, in, in, nullptr, nullptr, nlines);
+            named_bar_sync(1 + grp, NWG * 32);
+            if constexpr (NA == 1) {
+                apply_lines_gc<P1, 1, 1, TC::R, NWG, C, 1, OUT_GLOBAL>(wg, in, nullptr, nullptr, V + e0 * NPTS, nlines);
+            } else {
+                apply_lines_gc<P1, P1, 1, TC::R, NWG, C, 1, OUT_SMEM>(wg, in, in, nullptr, nullptr, nlines);
+                named_bar_sync(1 + grp, NWG * 32);
+                sq += apply_lines_gc<P1, P1, 0, TC::R, NWG, C, 2, OUT_GLOBAL, true>(wg, in, nullptr, nullptr,
+                                                                                      V + e0 * NPTS, nlines);
+            }
+            release_slot(empty0 + 8 * b, lane);
+        }
+    }
+    if (NA != 1 && ws != nullptr) block_partial(sq, ws + 8);
+}
+
+// Odd P1 >= BC_T3_MIN_P1 with constant-bank operators and 16-byte aligned U: the TMA ring
+// kernel (measured: DESIGN.md §4.1); BC_SF3_TMA=0 in the environment selects the
+// unbuffered kernel for A/B measurements (read once).
+#ifndef BC_T3_MIN_P1
+#define BC_T3_MIN_P1 13
+#endif
+#ifndef BC_T2_MIN_P1
+#define BC_T2_MIN_P1 5
+#endif
+static bool sf2_tma_enabled() {
+    static const bool on = [] {
+        const char* v = getenv("BC_SF2_TMA");
+        return !(v && v[0] == '0');
+    }();
+    return on;
+}
+static bool sf3_tma_enabled() {
+    static const bool on = [] {
+        const char* v = getenv("BC_SF3_TMA");
+        return !(v && v[0] == '0');
+    }();
+    return on;
+}
+
+template <int P1, int NA, int CS>
+int launch_sumfact_tma(int64_t N, const double* U, double* V, double* ws, cudaStream_t s) {
+    using TC = TmaSf3<P1, NA>;
+    static PerDevice<int> attr_dev;
+    int& attr = attr_dev.get();
+    if (!attr) {
+        cudaFuncSetAttribute(sumfact_tma_kernel<P1, NA, CS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)TC::SMEM);
+        attr = 1;
+    }
+    const int64_t ngroups = (N + TC::E - 1) / TC::E;
+    int grid = (int)imin64(ngroups, num_sms());
+    if (ws && grid > CHECK_MAX_PARTIALS) grid = CHECK_MAX_PARTIALS;
+    sumfact_tma_kernel<P1, NA, CS><<<grid, TC::NT, TC::SMEM, s>>>(N, U, V, ws);
+    const int st = launch_status();
+    op_slot_release(s, CS);
+    if (st || !ws) return st;
+    return run_check_finalize(grid, ws, s);
+}
+
 template <int P1, typename T>
 int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, T* V, double* ws, cudaStream_t s) {
     if constexpr (sizeof(T) == 8) {
@@ -692,6 +906,11 @@ int launch_sumfact3d(int64_t N, const T* A, const T* B, const T* C, const T* U, 
             const double* ops[3] = {A, B, C};
             int slot, st;
             if ((st = op_slot_acquire(s, ops, 3, P1, &slot))) return st;
+            if constexpr (P1 % 2 == 1 && TmaSf3<P1>::FITS && P1 >= BC_T3_MIN_P1) {
+                if (sf3_tma_enabled() && (reinterpret_cast<uintptr_t>(U) & 15) == 0)
+                    return slot == 0 ? launch_sumfact_tma<P1, P1, 0>(N, U, V, ws, s)
+                                     : launch_sumfact_tma<P1, P1, 1>(N, U, V, ws, s);
+            }
             return slot == 0 ? launch_sumfact3d_k<P1, T, 0>(N, A, B, C, U, V, ws, s)
                              : launch_sumfact3d_k<P1, T, 1>(N, A, B, C, U, V, ws, s);
         }
@@ -756,6 +975,11 @@ int launch_sumfact2d(int64_t N, const double* A, const double* B, const double* 
         const double* ops[2] = {A, B};
         int slot, st;
         if ((st = op_slot_acquire(s, ops, 2, P1, &slot))) return st;
+        if constexpr (P1 % 2 == 1 && TmaSf3<P1, 1>::FITS && P1 >= BC_T2_MIN_P1) {
+            if (sf2_tma_enabled() && (reinterpret_cast<uintptr_t>(U) & 15) == 0)
+                return slot == 0 ? launch_sumfact_tma<P1, 1, 0>(N, U, V, nullptr, s)
+                                 : launch_sumfact_tma<P1, 1, 1>(N, U, V, nullptr, s);
+        }
         return slot == 0 ? launch_sumfact2d_k<P1, 0>(N, A, B, U, V, s) : launch_sumfact2d_k<P1, 1>(N, A, B, U, V, s);
     }
     return launch_sumfact2d_k<P1, -1>(N, A, B, U, V, s);
@@ -804,6 +1028,139 @@ local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __rest
     });
 }
 
+// ------------------------------------------------------------ local_grad3, TMA element ring
+// Warp-specialised persistent form of local_grad3_kernel (odd P1, constant-bank D), the
+// same ring as sumfact_tma_kernel plus a storer warp:
+//   consumers (group of NWG warps per item): us and ut stored from registers (coalesced),
+//     group barrier, ur formed in place in the slot, generic->async proxy fence, one
+//     `done` arrive per warp;
+//   storer (one thread): per item in order, waits `done`, writes ur with a 1-D bulk copy
+//     shared -> global (the values outside its 16-byte aligned interior by plain stores),
+//     and releases the previous item's slot once that copy has finished reading it.
+// The loader and the storer run asynchronously to the consumers, so the consumers neither
+// wait for element data nor issue the ur copy-out (the unbuffered kernel's 24%
+// long-scoreboard and 19% barrier stalls).
+#ifndef BC_L3_E
+#define BC_L3_E 0  // 0: max(1, elements whose lines fill the group's 32 NWG R lanes)
+#endif
+#ifndef BC_L3_NB
+#define BC_L3_NB 10
+#endif
+#ifndef BC_L3_NG
+#define BC_L3_NG 5
+#endif
+#ifndef BC_L3_NWG
+#define BC_L3_NWG 2
+#endif
+#ifndef BC_L3_R
+#define BC_L3_R 3
+#endif
+#ifndef BC_L3_NUNR
+#define BC_L3_NUNR 1
+#endif
+template <int P1>
+using TmaLg3 = Ring<P1 * P1 * P1,
+                    (BC_L3_E ? BC_L3_E : (32 * BC_L3_NWG * BC_L3_R / (P1 * P1) > 1 ? 32 * BC_L3_NWG * BC_L3_R / (P1 * P1) : 1)),
+                    BC_L3_NB, BC_L3_NG, BC_L3_NWG, BC_L3_R, 2>;
+
+template <int P1, int CS>
+__global__ void __launch_bounds__(TmaLg3<P1>::NT, 1)
+local_grad3_tma_kernel(int64_t N, const double* __restrict__ U, double* __restrict__ ur, double* __restrict__ us,
+                       double* __restrict__ ut) {
+    using TC = TmaLg3<P1>;
+    constexpr int E = TC::E, NB = TC::NB, NG = TC::NG, NWG = TC::NWG, NPTS = TC::NPTS;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    double* slots = reinterpret_cast<double*>(smem_raw);
+    const uint32_t full0 = smem_u32(smem_raw + (size_t)NB * TC::SLOT * 8), empty0 = full0 + 8 * NB,
+                   done0 = empty0 + 8 * NB;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int b = 0; b < NB; ++b) {
+            mbar_init(full0 + 8 * b, 1);
+            mbar_init(empty0 + 8 * b, 1);
+            mbar_init(done0 + 8 * b, NWG);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const int64_t ngroups = (N + E - 1) / E;
+    const int64_t nitems = ngroups > blockIdx.x ? (ngroups - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    if (warp == NG * NWG) {
+        if (lane == 0) ring_loader<TC>(N, U, slots, full0, empty0, nitems);
+    } else if (warp == NG * NWG + 1) {
+        if (lane == 0) {
+            for (int64_t j = 0; j < nitems; ++j) {
+                const int b = (int)(j % NB);
+                mbar_wait(done0 + 8 * b, (int)((j / NB) & 1));
+                const int64_t e0 = (blockIdx.x + j * gridDim.x) * E;
+                const int n = (int)imin64(E, N - e0) * NPTS;
+                const int h = item_lead(U + e0 * NPTS);  // == item_lead(ur + e0 * NPTS)
+                const double* in = slots + (size_t)b * TC::SLOT + h;
+                double* dst = ur + e0 * NPTS;
+                const int m = (n - h) & ~1;  // values in the 16-byte aligned interior [h, h + m)
+                if (h) dst[0] = in[0];
+                if (h + m < n) dst[n - 1] = in[n - 1];
+                if (m) bulk_store(dst + h, smem_u32(in + h), (uint32_t)m * 8u);
+                bulk_commit();
+                if (j > 0) {
+                    bulk_wait_read<1>();  // item j-1's copy has read its slot
+                    fence_proxy_async();
+                    mbar_arrive(empty0 + 8 * (int)((j - 1) % NB));
+                }
+            }
+            bulk_wait<0>();
+        }
+    } else {
+        constexpr int C = CS;
+        const int grp = warp / NWG, wg = warp - grp * NWG;
+        for (int64_t j = grp; j < nitems; j += NG) {
+            const int b = (int)(j % NB);
+            ring_wait_full<NB>(full0, empty0, b, j);
+            const int64_t e0 = (blockIdx.x + j * gridDim.x) * E, gbase = e0 * NPTS;
+            const int nlines = (int)imin64(E, N - e0) * P1 * P1;
+            double* in = slots + (size_t)b * TC::SLOT + item_lead(U + gbase);
+            constexpr int U = BC_L3_NUNR;
+            apply_lines_gc<P1, P1, 1, TC::R, NWG, C, 0, OUT_GLOBAL, false, false, U>(wg, in, nullptr, nullptr,
+                                                                                   us + gbase, nlines);
+            apply_lines_gc<P1, P1, 0, TC::R, NWG, C, 0, OUT_GLOBAL, false, false, U>(wg, in, nullptr, nullptr,
+                                                                                   ut + gbase, nlines);
+            named_bar_sync(1 + grp, NWG * 32);  // every read of the item precedes ur's in-place writes
+            apply_lines_gc<P1, P1, 2, TC::R, NWG, C, 0, OUT_SMEM, false, false, U>(wg, in, in, nullptr, nullptr, nlines);
+            fence_proxy_async();  // ur (generic writes) is read next by the storer's bulk copy
+            __syncwarp();
+            if (lane == 0) mbar_arrive(done0 + 8 * b);
+        }
+    }
+}
+
+#ifndef BC_L3_MIN_P1
+#define BC_L3_MIN_P1 5
+#endif
+static bool lg3_tma_enabled() {
+    static const bool on = [] {
+        const char* v = getenv("BC_LG3_TMA");
+        return !(v && v[0] == '0');
+    }();
+    return on;
+}
+
+template <int P1, int CS>
+int launch_local_grad3_tma(int64_t N, const double* U, double* ur, double* us, double* ut, cudaStream_t s) {
+    using TC = TmaLg3<P1>;
+    static PerDevice<int> attr_dev;
+    int& attr = attr_dev.get();
+    if (!attr) {
+        cudaFuncSetAttribute(local_grad3_tma_kernel<P1, CS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)TC::SMEM);
+        attr = 1;
+    }
+    const int grid = (int)imin64((N + TC::E - 1) / TC::E, num_sms());
+    local_grad3_tma_kernel<P1, CS><<<grid, TC::NT, TC::SMEM, s>>>(N, U, ur, us, ut);
+    const int st = launch_status();
+    op_slot_release(s, CS);
+    return st;
+}
+
 template <int P1, int CS>
 int launch_local_grad3_k(int64_t N, const double* D, const double* U, double* ur, double* us, double* ut,
                          cudaStream_t s) {
@@ -824,6 +1181,13 @@ int launch_local_grad3(int64_t N, const double* D, const double* U, double* ur, 
     if (N >= OPS_CONST_MIN_N) {
         int slot, st;
         if ((st = op_slot_acquire(s, &D, 1, P1, &slot))) return st;
+        // odd P1 (unpadded smem layout) except 11, where a one-element item's 121 lines fill
+        // 121 of a group's 192 lanes (measured: ring 0.74 vs unbuffered 0.86 of HBM)
+        if constexpr (P1 % 2 == 1 && TmaLg3<P1>::FITS && P1 >= BC_L3_MIN_P1 && P1 != 11) {
+            if (lg3_tma_enabled() && ((reinterpret_cast<uintptr_t>(U) | reinterpret_cast<uintptr_t>(ur)) & 15) == 0)
+                return slot == 0 ? launch_local_grad3_tma<P1, 0>(N, U, ur, us, ut, s)
+                                 : launch_local_grad3_tma<P1, 1>(N, U, ur, us, ut, s);
+        }
         return slot == 0 ? launch_local_grad3_k<P1, 0>(N, D, U, ur, us, ut, s)
                          : launch_local_grad3_k<P1, 1>(N, D, U, ur, us, ut, s);
     }

@@ -205,3 +205,57 @@ def test_constant_bank_operators_two_streams_and_graph(bc):
     torch.cuda.synchronize()
     for i, (out, ref) in enumerate(zip(gouts, refs)):
         assert np.array_equal(to_host(out), ref), f"graph call {i}"
+
+
+@pytest.mark.parametrize("P1", [13])
+def test_sumfact3d_tma_ring_integer_bitwise(bc, P1):
+    """The warp-specialised TMA element-ring kernel (csrc/spectral.cu sumfact3d_tma_kernel,
+    odd P1 >= 9, N >= 128, 16-byte aligned U): N = 148 CTAs x 2 elements x 6 slots x 2 + 1,
+    so every CTA's ring wraps at least twice and the last item is ragged (one element, an
+    odd number of values: bulk copy + the plain-copied last value); every element bitwise
+    vs the oracle (items alternately start on and 8 bytes off a 16-byte boundary); then
+    N + 1 elements (even: no plain-copied value) with the fused check scalar."""
+    A, B, C = (syn.tensor(t, (P1, P1), kind=syn.KIND_INT) for t in (2, 3, 4))
+    N = 148 * 2 * 6 * 2 + 1
+    U = syn.tensor(1, (N + 1, P1, P1, P1), kind=syn.KIND_INT)
+    Ud = to_dev(U)
+    Ad, Bd, Cd = to_dev(A), to_dev(B), to_dev(C)
+    ref = oracle.sumfact3d(A, B, C, U)
+    V = bc.sumfact3d(Ad, Bd, Cd, Ud[:N], out=poisoned_like(Ud[:N]))
+    assert np.array_equal(to_host(V), ref[:N]), f"P1={P1} N={N}"
+    ws = torch.full((1024,), float("nan"), dtype=torch.float64, device="cuda")
+    V2 = bc.sumfact3d(Ad, Bd, Cd, Ud, out=poisoned_like(Ud), check_ws=ws)
+    assert np.array_equal(to_host(V2), ref)
+    s = oracle.sumsq(ref)
+    assert abs(ws[0].item() - s) <= 1e-12 * s
+
+
+@pytest.mark.parametrize("N", [128, 129, 148 * 2 * 5 * 2 + 1, 148 * 2 * 5 * 3 + 2])
+def test_local_grad3_tma_ring_integer_bitwise(bc, N):
+    """The warp-specialised TMA element-ring local_grad3 (csrc/spectral.cu
+    local_grad3_tma_kernel, P1 = 13, N >= 128, 16-byte aligned U and ur): rings that do not
+    wrap, wrap twice and three times; items alternately on and 8 bytes off a 16-byte
+    boundary, so ur's bulk store writes its first/last value by plain stores; an odd N
+    (the last item's final value plain-copied in); ur/us/ut every element bitwise."""
+    P1 = 13
+    D = syn.tensor(6, (P1, P1), kind=syn.KIND_INT)
+    U = syn.tensor(1, (N, P1, P1, P1), kind=syn.KIND_INT)
+    Ud = to_dev(U)
+    outs = tuple(poisoned_like(Ud) for _ in range(3))
+    got = bc.local_grad3(to_dev(D), Ud, out=outs)
+    for g, r, name in zip(got, oracle.local_grad3(D, U), ("ur", "us", "ut")):
+        assert np.array_equal(to_host(g), r), f"{name} N={N}"
+
+
+@pytest.mark.parametrize("P1", [5, 9, 13])
+@pytest.mark.parametrize("N", [128, 148 * 40 * 12 * 2 + 1])
+def test_sumfact2d_tma_ring_integer_bitwise(bc, P1, N):
+    """The TMA element-ring sumfact2d (csrc/spectral.cu sumfact_tma_kernel<P1, 1>, items of
+    32 NWG R / P1 2-D elements, where enabled; the other P1 run the unbuffered kernel): a
+    ring that does not wrap and one that wraps at least twice with a ragged last item; every
+    element bitwise vs the oracle."""
+    A, B = (syn.tensor(t, (P1, P1), kind=syn.KIND_INT) for t in (2, 3))
+    U = syn.tensor(1, (N, P1, P1), kind=syn.KIND_INT)
+    Ud = to_dev(U)
+    V = bc.sumfact2d(to_dev(A), to_dev(B), Ud, out=poisoned_like(Ud))
+    assert np.array_equal(to_host(V), oracle.sumfact2d(A, B, U)), f"P1={P1} N={N}"

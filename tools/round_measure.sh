@@ -11,7 +11,7 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/
     python bench.py --no-cpu --no-e2e --no-configs --steps 2 --warmup 3 > /dev/null 2> $OUT/launches.err
 # (kernel regex, launches to skip): one launch each; ccsdt_tma_kernel twice (a d1 launch,
 # then a d2 launch: 8 d1 then 8 d2 launches per step)
-for ks in local_grad3_kernel:2 sumfact3d_kernel:2 sumfact2d_kernel:2 ccsdt_tma_kernel:2 ccsdt_tma_kernel:10; do
+for ks in local_grad3_tma_kernel:2 sumfact_tma_kernel:2 sumfact_tma_kernel:3 ccsdt_tma_kernel:2 ccsdt_tma_kernel:10; do
   k=${ks%%:*}; s=${ks##*:}
   ncu --set full --clock-control none --import-source on -k regex:$k -s $s -c 1 -o $OUT/prof_${k}_s$s -f \
       python bench.py --no-cpu --no-e2e --no-configs --steps 1 --warmup 3 > /dev/null 2> $OUT/prof_$k.err

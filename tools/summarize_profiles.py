@@ -100,8 +100,12 @@ for f in sorted(os.listdir(G)):
         return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(u, 1)
     if "dram__bytes_read.sum" in d:
         base = name.split("(")[0].split("<")[0].replace("void ", "").replace("bc::", "").strip()
-        kn = {"local_grad3_kernel": "local_grad3", "sumfact3d_kernel": "sumfact3d", "sumfact2d_kernel": "sumfact2d",
+        kn = {"local_grad3_kernel": "local_grad3", "local_grad3_tma_kernel": "local_grad3",
+              "sumfact3d_kernel": "sumfact3d", "sumfact2d_kernel": "sumfact2d",
               "ccsdt_tma_kernel": "ccsdt_tma"}.get(base, base)
+        if base == "sumfact_tma_kernel":  # <P1, NA, CS>: NA = 1 is the 2-D form
+            targs = [a.replace("(int)", "").strip() for a in name.split("<", 1)[1].split(">", 1)[0].split(",")]
+            kn = "sumfact2d" if targs[1] == "1" else "sumfact3d"
         tb = gb("dram__bytes_read.sum") + gb("dram__bytes_write.sum")
         n_elem = cfg.get("n_elem", cfg.get("n_elem_per_gpu"))
         if kn == "ccsdt_tma":
