@@ -353,6 +353,9 @@ struct TmaMaps {
 #ifndef BC_EXP16_NOFLUSH
 #define BC_EXP16_NOFLUSH 0  // timing experiments only: skip the class flushes of the 16-cube kernel
 #endif
+#ifndef BC_EXP16_NOTMA
+#define BC_EXP16_NOTMA 0  // timing experiments only: no operand copies (the ring still cycles)
+#endif
 #ifndef BC_EXP16_NOSTORE
 #define BC_EXP16_NOSTORE 0  // timing experiments only: skip the store / re-seed of the 16-cube kernel
 #endif
@@ -625,9 +628,13 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
                 const uint32_t full = bar_full + 8 * slot;
                 if (lane == 0) {
                     mbar_wait(bar_empty + 8 * slot, ((g / NS) & 1) ^ 1);
-                    mbar_expect_tx(full, TG::STAGE_BYTES);
+                    if (BC_EXP16_NOTMA)  // timing experiment only (stale operands)
+                        mbar_arrive(full);
+                    else
+                        mbar_expect_tx(full, TG::STAGE_BYTES);
                 }
                 __syncwarp();
+                if (BC_EXP16_NOTMA) continue;
                 const int k0 = kc_i * KC;
                 if (++kc_i == nchunk) kc_i = 0;
                 const int e_cur = e;

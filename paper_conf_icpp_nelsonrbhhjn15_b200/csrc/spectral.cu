@@ -723,21 +723,32 @@ int launch_sumfact3d_k(int64_t N, const T* A, const T* B, const T* C, const T* U
 #ifndef BC_T3_R
 #define BC_T3_R 3
 #endif
+#ifndef BC_T3S_NB
+#define BC_T3S_NB 10
+#endif
+#ifndef BC_T3S_NG
+#define BC_T3S_NG 6
+#endif
+#ifndef BC_T3S_R
+#define BC_T3S_R 4
+#endif
 // Ring geometry: items of E elements of NPTS values, NB slots, NG x NWG consumer warps plus
 // XW service warps (loader; storer).
-template <int NPTS_, int E_, int NB_, int NG_, int NWG_, int R_, int XW>
+template <int NPTS_, int E_, int NB_, int NG_, int NWG_, int R_, int XW, int NF_ = 1>
 struct Ring {
-    static constexpr int E = E_, NB = NB_, NG = NG_, NWG = NWG_, R = R_, NPTS = NPTS_;
-    // doubles per slot: an item may start 8 bytes past a 16-byte boundary (odd E x odd
-    // NPTS); its copy then starts one value early and may end one value late (16-byte
-    // aligned, multiple-of-16 bulk copies), so a slot holds E * NPTS + 2 values
-    static constexpr int SLOT = (E * NPTS + 2 + 1) & ~1;
+    static constexpr int E = E_, NB = NB_, NG = NG_, NWG = NWG_, R = R_, NPTS = NPTS_, NF = NF_;
+    // doubles per field of a slot: an item may start 8 bytes past a 16-byte boundary (odd
+    // E x odd NPTS); its copy then starts one value early and may end one value late
+    // (16-byte aligned, multiple-of-16 bulk copies), so a field holds E * NPTS + 2 values.
+    // A slot holds NF fields (local_grad3_t: ur, us, ut).
+    static constexpr int SUB = (E * NPTS + 2 + 1) & ~1;
+    static constexpr int SLOT = NF * SUB;
     static constexpr int NT = 32 * (NG * NWG + XW);
     static constexpr size_t SMEM = (size_t)NB * SLOT * 8 + 3 * NB * 8;
     static constexpr bool FITS = SMEM <= 227 * 1024;
     static_assert(NB > NG, "ring_wait_full needs more slots than consumer groups");
 };
-// 2-D (sumfact2d) ring: items of E2 elements of P1^2 values (26 x 169 = 2 x 13^3 at P1 = 13)
+// 2-D (sumfact2d) ring: items of E2 elements of P1^2 values
 #ifndef BC_T2_E
 #define BC_T2_E 0  // 0: as many elements as fill the group's 32 NWG R lanes' lines
 #endif
@@ -756,7 +767,11 @@ struct Ring {
 template <int P1, int NA = P1>
 using TmaSf3 = typename std::conditional<
     NA == 1, Ring<P1 * P1, (BC_T2_E ? BC_T2_E : 32 * BC_T2_NWG * BC_T2_R / P1), BC_T2_NB, BC_T2_NG, BC_T2_NWG, BC_T2_R, 1>,
-    Ring<P1 * P1 * P1, BC_T3_E, BC_T3_NB, BC_T3_NG, BC_T3_NWG, BC_T3_R, 1>>::type;
+    typename std::conditional<
+        P1 == 13, Ring<P1 * P1 * P1, BC_T3_E, BC_T3_NB, BC_T3_NG, BC_T3_NWG, BC_T3_R, 1>,
+        // other odd P1: items of max(1, 192 / P1^2) elements on 2-warp groups
+        Ring<P1 * P1 * P1, (64 * BC_T3S_R / (P1 * P1) > 1 ? 64 * BC_T3S_R / (P1 * P1) : 1), BC_T3S_NB, BC_T3S_NG, 2,
+             BC_T3S_R, 1>>::type>::type;
 
 // item j of this CTA: elements [e0, e0 + ne); its first value sits at slot + item_lead
 __device__ __forceinline__ int item_lead(const double* p) { return (int)((reinterpret_cast<uintptr_t>(p) >> 3) & 1); }
@@ -768,24 +783,35 @@ __device__ __forceinline__ int item_lead(const double* p) { return (int)((reinte
 // expect_tx.  A slot is refilled after its empty barrier's previous phase completed.
 template <class RG>
 __device__ __forceinline__ void ring_loader(int64_t N, const double* __restrict__ U, double* slots, uint32_t full0,
-                                            uint32_t empty0, int64_t nitems) {
+                                            uint32_t empty0, int64_t nitems, const double* __restrict__ U1 = nullptr,
+                                            const double* __restrict__ U2 = nullptr) {
+    const double* F[3] = {U, U1, U2};
     for (int64_t j = 0; j < nitems; ++j) {
         const int b = (int)(j % RG::NB);
         const int64_t use = j / RG::NB;
         if (use > 0) mbar_wait(empty0 + 8 * b, (int)((use - 1) & 1));
         const int64_t e0 = (blockIdx.x + j * gridDim.x) * RG::E;
         const int ne = (int)imin64(RG::E, N - e0);
-        const double* src = U + e0 * RG::NPTS;
-        const int lead = item_lead(src);
-        const int tot = lead + ne * RG::NPTS;
-        int nv = (tot + 1) >> 1;
-        double* dst = slots + (size_t)b * RG::SLOT;
-        if ((tot & 1) && e0 + ne == N) {
-            nv = tot >> 1;
-            dst[tot - 1] = src[tot - 1 - lead];
+        int nv[RG::NF], bytes = 0;
+#pragma unroll
+        for (int f = 0; f < RG::NF; ++f) {
+            const double* src = F[f] + e0 * RG::NPTS;
+            const int lead = item_lead(src);
+            const int tot = lead + ne * RG::NPTS;
+            nv[f] = (tot + 1) >> 1;
+            if ((tot & 1) && e0 + ne == N) {
+                nv[f] = tot >> 1;
+                slots[(size_t)b * RG::SLOT + f * RG::SUB + tot - 1] = src[tot - 1 - lead];
+            }
+            bytes += nv[f] * 16;
         }
-        mbar_expect_tx(full0 + 8 * b, nv * 16);
-        bulk_load(smem_u32(dst), src - lead, (uint32_t)nv * 16u, full0 + 8 * b);
+        mbar_expect_tx(full0 + 8 * b, bytes);
+#pragma unroll
+        for (int f = 0; f < RG::NF; ++f) {
+            const double* src = F[f] + e0 * RG::NPTS;
+            bulk_load(smem_u32(slots + (size_t)b * RG::SLOT + f * RG::SUB), src - item_lead(src),
+                      (uint32_t)nv[f] * 16u, full0 + 8 * b);
+        }
     }
 }
 
@@ -859,7 +885,7 @@ sumfact_tma_kernel(int64_t N, const double* __restrict__ U, double* __restrict__
 // kernel (measured: DESIGN.md §4.1); BC_SF3_TMA=0 in the environment selects the
 // unbuffered kernel for A/B measurements (read once).
 #ifndef BC_T3_MIN_P1
-#define BC_T3_MIN_P1 13
+#define BC_T3_MIN_P1 5
 #endif
 #ifndef BC_T2_MIN_P1
 #define BC_T2_MIN_P1 5
@@ -1058,6 +1084,9 @@ local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __rest
 #ifndef BC_L3_NUNR
 #define BC_L3_NUNR 1
 #endif
+#ifndef BC_L3_EAGER
+#define BC_L3_EAGER 1  // storer releases a slot as soon as its ur copy has read it
+#endif
 template <int P1>
 using TmaLg3 = Ring<P1 * P1 * P1,
                     (BC_L3_E ? BC_L3_E : (32 * BC_L3_NWG * BC_L3_R / (P1 * P1) > 1 ? 32 * BC_L3_NWG * BC_L3_R / (P1 * P1) : 1)),
@@ -1102,7 +1131,11 @@ local_grad3_tma_kernel(int64_t N, const double* __restrict__ U, double* __restri
                 if (h + m < n) dst[n - 1] = in[n - 1];
                 if (m) bulk_store(dst + h, smem_u32(in + h), (uint32_t)m * 8u);
                 bulk_commit();
-                if (j > 0) {
+                if constexpr (BC_L3_EAGER) {
+                    bulk_wait_read<0>();  // this item's copy has read its slot: release it now
+                    fence_proxy_async();
+                    mbar_arrive(empty0 + 8 * b);
+                } else if (j > 0) {
                     bulk_wait_read<1>();  // item j-1's copy has read its slot
                     fence_proxy_async();
                     mbar_arrive(empty0 + 8 * (int)((j - 1) % NB));
@@ -1253,6 +1286,105 @@ local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __re
     }
 }
 
+// ------------------------------------------------------------ local_grad3_t, TMA element ring
+// The ring of local_grad3 with three input fields per item (ur, us, ut in one slot, one
+// full barrier for the three bulk copies): r stage in place on ur, group barrier, s stage
+// into us adding ur, group barrier, t stage to U (global, coalesced) adding us; the same
+// (r + s) + t order as local_grad3_t_kernel.  Items of one element (3 x 17.6 KB at P1 = 13).
+#ifndef BC_LT_NB
+#define BC_LT_NB 4
+#endif
+#ifndef BC_LT_NG
+#define BC_LT_NG 3
+#endif
+#ifndef BC_LT_NWG
+#define BC_LT_NWG 3
+#endif
+#ifndef BC_LT_R
+#define BC_LT_R 3
+#endif
+#ifndef BC_LT13_R
+#define BC_LT13_R 2  // P1 = 13: 169 lines on 3 warps x 64 lanes (R = 3 leaves one warp idle)
+#endif
+template <int P1, int LR = (P1 == 13 ? BC_LT13_R : BC_LT_R)>
+using TmaLgT = Ring<P1 * P1 * P1,
+                    (32 * BC_LT_NWG * LR / (P1 * P1) > 1 ? 32 * BC_LT_NWG * LR / (P1 * P1) : 1),
+                    BC_LT_NB, BC_LT_NG, BC_LT_NWG, LR, 1, 3>;
+
+template <int P1, int CS>
+__global__ void __launch_bounds__(TmaLgT<P1>::NT, 1)
+local_grad3_t_tma_kernel(int64_t N, const double* __restrict__ ur, const double* __restrict__ us,
+                         const double* __restrict__ ut, double* __restrict__ U) {
+    using TC = TmaLgT<P1>;
+    constexpr int E = TC::E, NB = TC::NB, NG = TC::NG, NWG = TC::NWG, NPTS = TC::NPTS;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    double* slots = reinterpret_cast<double*>(smem_raw);
+    const uint32_t full0 = smem_u32(smem_raw + (size_t)NB * TC::SLOT * 8), empty0 = full0 + 8 * NB;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int b = 0; b < NB; ++b) {
+            mbar_init(full0 + 8 * b, 1);
+            mbar_init(empty0 + 8 * b, NWG);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const int64_t ngroups = (N + E - 1) / E;
+    const int64_t nitems = ngroups > blockIdx.x ? (ngroups - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    if (warp == NG * NWG) {
+        if (lane == 0) ring_loader<TC>(N, ur, slots, full0, empty0, nitems, us, ut);
+    } else {
+        constexpr int C = CS;
+        const int grp = warp / NWG, wg = warp - grp * NWG;
+        for (int64_t j = grp; j < nitems; j += NG) {
+            const int b = (int)(j % NB);
+            ring_wait_full<NB>(full0, empty0, b, j);
+            const int64_t e0 = (blockIdx.x + j * gridDim.x) * E, gbase = e0 * NPTS;
+            const int nlines = (int)imin64(E, N - e0) * P1 * P1;
+            double* slot = slots + (size_t)b * TC::SLOT;
+            double* bR = slot + item_lead(ur + gbase);
+            double* bS = slot + TC::SUB + item_lead(us + gbase);
+            double* bT = slot + 2 * TC::SUB + item_lead(ut + gbase);
+            apply_lines_gc<P1, P1, 2, TC::R, NWG, C, 0, OUT_SMEM, false, true>(wg, bR, bR, nullptr, nullptr, nlines);
+            named_bar_sync(1 + grp, NWG * 32);
+            apply_lines_gc<P1, P1, 1, TC::R, NWG, C, 0, OUT_SMEM_ADD, false, true>(wg, bS, bS, bR, nullptr, nlines);
+            named_bar_sync(1 + grp, NWG * 32);
+            apply_lines_gc<P1, P1, 0, TC::R, NWG, C, 0, OUT_GLOBAL_ADD, false, true>(wg, bT, nullptr, bS, U + gbase,
+                                                                                     nlines);
+            release_slot(empty0 + 8 * b, lane);
+        }
+    }
+}
+
+#ifndef BC_LT_MIN_P1
+#define BC_LT_MIN_P1 5
+#endif
+static bool lg3t_tma_enabled() {
+    static const bool on = [] {
+        const char* v = getenv("BC_LG3T_TMA");
+        return !(v && v[0] == '0');
+    }();
+    return on;
+}
+
+template <int P1, int CS>
+int launch_local_grad3_t_tma(int64_t N, const double* ur, const double* us, const double* ut, double* U,
+                             cudaStream_t s) {
+    using TC = TmaLgT<P1>;
+    static PerDevice<int> attr_dev;
+    int& attr = attr_dev.get();
+    if (!attr) {
+        cudaFuncSetAttribute(local_grad3_t_tma_kernel<P1, CS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)TC::SMEM);
+        attr = 1;
+    }
+    const int grid = (int)imin64((N + TC::E - 1) / TC::E, num_sms());
+    local_grad3_t_tma_kernel<P1, CS><<<grid, TC::NT, TC::SMEM, s>>>(N, ur, us, ut, U);
+    const int st = launch_status();
+    op_slot_release(s, CS);
+    return st;
+}
+
 template <int P1, int CS>
 int launch_local_grad3_t_k(int64_t N, const double* D, const double* ur, const double* us, const double* ut,
                            double* U, cudaStream_t s) {
@@ -1273,6 +1405,13 @@ int launch_local_grad3_t(int64_t N, const double* D, const double* ur, const dou
     if (N >= OPS_CONST_MIN_N) {
         int slot, st;
         if ((st = op_slot_acquire(s, &D, 1, P1, &slot))) return st;
+        if constexpr (P1 % 2 == 1 && TmaLgT<P1>::FITS && P1 >= BC_LT_MIN_P1) {
+            if (lg3t_tma_enabled() &&
+                ((reinterpret_cast<uintptr_t>(ur) | reinterpret_cast<uintptr_t>(us) | reinterpret_cast<uintptr_t>(ut)) &
+                 15) == 0)
+                return slot == 0 ? launch_local_grad3_t_tma<P1, 0>(N, ur, us, ut, U, s)
+                                 : launch_local_grad3_t_tma<P1, 1>(N, ur, us, ut, U, s);
+        }
         return slot == 0 ? launch_local_grad3_t_k<P1, 0>(N, D, ur, us, ut, U, s)
                          : launch_local_grad3_t_k<P1, 1>(N, D, ur, us, ut, U, s);
     }

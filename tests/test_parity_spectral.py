@@ -259,3 +259,15 @@ def test_sumfact2d_tma_ring_integer_bitwise(bc, P1, N):
     Ud = to_dev(U)
     V = bc.sumfact2d(to_dev(A), to_dev(B), Ud, out=poisoned_like(Ud))
     assert np.array_equal(to_host(V), oracle.sumfact2d(A, B, U)), f"P1={P1} N={N}"
+
+
+@pytest.mark.parametrize("P1", [5, 9, 11, 13])
+def test_local_grad3_t_tma_ring_integer_bitwise(bc, P1):
+    """The TMA ring local_grad3_t (csrc/spectral.cu local_grad3_t_tma_kernel: three input
+    fields per slot): N large enough for every CTA's 4-slot ring to wrap several times, odd
+    (ragged last item with plain-copied final values); every element bitwise."""
+    N = 148 * 4 * 3 * max(1, 192 // (P1 * P1)) + 1
+    D = syn.tensor(6, (P1, P1), kind=syn.KIND_INT)
+    ur, us, ut = (syn.tensor(t, (N, P1, P1, P1), kind=syn.KIND_INT) for t in (7, 8, 9))
+    got = bc.local_grad3_t(to_dev(D), to_dev(ur), to_dev(us), to_dev(ut), out=poisoned_like(to_dev(ur)))
+    assert np.array_equal(to_host(got), oracle.local_grad3_t(D, ur, us, ut)), f"P1={P1} N={N}"

@@ -95,3 +95,19 @@ def test_ring_local_grad3_repeat_bitwise(bc, P1):
     idx = torch.from_numpy(els).cuda()
     for g, r in zip(refs, oracle.local_grad3(D, int_elements(syn.TID["U"], P1, els))):
         assert np.array_equal(g[idx].cpu().numpy(), r)
+
+
+@pytest.mark.parametrize("P1", [5, 9, 13])
+def test_ring_local_grad3_t_repeat_bitwise(bc, P1):
+    N = (1 << 27) // (P1 ** 3 * 8) + 1
+    D = syn.tensor(6, (P1, P1), kind=syn.KIND_INT)
+    dD = torch.from_numpy(D).cuda()
+    ins = [int_field(bc, (N, P1, P1, P1), t) for t in (7, 8, 9)]
+    U = torch.empty_like(ins[0])
+    bc.local_grad3_t(dD, *ins, out=U)
+    torch.cuda.synchronize()
+    (Ur,) = repeat_equal(lambda: bc.local_grad3_t(dD, *ins, out=U), [U])
+    els = sample(N, 30 + P1)
+    got = Ur[torch.from_numpy(els).cuda()].cpu().numpy()
+    ref = oracle.local_grad3_t(D, *(int_elements(t, P1, els) for t in (7, 8, 9)))
+    assert np.array_equal(got, ref)

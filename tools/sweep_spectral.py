@@ -41,7 +41,10 @@ for p in ps:
         ("local_grad3", lambda: bc.local_grad3(D, U, out=outs), 32 * P1 ** 3 * N, 6 * P1 ** 4 * N),
         ("sumfact3d", lambda: bc.sumfact3d(A, A, A, U, out=V), 16 * P1 ** 3 * N, 6 * P1 ** 4 * N),
         ("sumfact2d", lambda: bc.sumfact2d(A, A, U2, out=V2), 16 * P1 ** 3 * N, 4 * P1 ** 3 * N * P1),
+        ("local_grad3_t", lambda: bc.local_grad3_t(D, *outs, out=V), 32 * P1 ** 3 * N, 6 * P1 ** 4 * N + 2 * P1 ** 3 * N),
     ):
+        if os.environ.get("SWEEP_ONLY") and name not in os.environ["SWEEP_ONLY"].split(","):
+            continue
         ms = timeit(fn)
         res[name] = {"ms": round(ms, 4), "hbm_frac": round(by / ms / 1e6 / HBM, 3), "tflops": round(fl / ms / 1e9, 2)}
     print(json.dumps({"lib": os.path.basename(bc.LIB_PATH), "p": p, "N": N, **res}), flush=True)
