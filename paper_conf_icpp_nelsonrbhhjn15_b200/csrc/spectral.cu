@@ -781,7 +781,7 @@ __device__ __forceinline__ int item_lead(const double* p) { return (int)((reinte
 // would read past the field's end (the last item only), the final value is copied by a
 // plain load/store instead, ordered before the consumers' reads by the release of
 // expect_tx.  A slot is refilled after its empty barrier's previous phase completed.
-template <class RG>
+template <class RG, int NL = RG::NF>
 __device__ __forceinline__ void ring_loader(int64_t N, const double* __restrict__ U, double* slots, uint32_t full0,
                                             uint32_t empty0, int64_t nitems, const double* __restrict__ U1 = nullptr,
                                             const double* __restrict__ U2 = nullptr) {
@@ -792,9 +792,9 @@ __device__ __forceinline__ void ring_loader(int64_t N, const double* __restrict_
         if (use > 0) mbar_wait(empty0 + 8 * b, (int)((use - 1) & 1));
         const int64_t e0 = (blockIdx.x + j * gridDim.x) * RG::E;
         const int ne = (int)imin64(RG::E, N - e0);
-        int nv[RG::NF], bytes = 0;
+        int nv[NL], bytes = 0;
 #pragma unroll
-        for (int f = 0; f < RG::NF; ++f) {
+        for (int f = 0; f < NL; ++f) {
             const double* src = F[f] + e0 * RG::NPTS;
             const int lead = item_lead(src);
             const int tot = lead + ne * RG::NPTS;
@@ -807,7 +807,7 @@ __device__ __forceinline__ void ring_loader(int64_t N, const double* __restrict_
         }
         mbar_expect_tx(full0 + 8 * b, bytes);
 #pragma unroll
-        for (int f = 0; f < RG::NF; ++f) {
+        for (int f = 0; f < NL; ++f) {
             const double* src = F[f] + e0 * RG::NPTS;
             bulk_load(smem_u32(slots + (size_t)b * RG::SLOT + f * RG::SUB), src - item_lead(src),
                       (uint32_t)nv[f] * 16u, full0 + 8 * b);

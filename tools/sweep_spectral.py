@@ -42,9 +42,15 @@ for p in ps:
         ("sumfact3d", lambda: bc.sumfact3d(A, A, A, U, out=V), 16 * P1 ** 3 * N, 6 * P1 ** 4 * N),
         ("sumfact2d", lambda: bc.sumfact2d(A, A, U2, out=V2), 16 * P1 ** 3 * N, 4 * P1 ** 3 * N * P1),
         ("local_grad3_t", lambda: bc.local_grad3_t(D, *outs, out=V), 32 * P1 ** 3 * N, 6 * P1 ** 4 * N + 2 * P1 ** 3 * N),
+        ("ax_e", "ax_e", 64 * P1 ** 3 * (N // 4), 12 * P1 ** 4 * (N // 4) + 17 * P1 ** 3 * (N // 4)),
     ):
         if os.environ.get("SWEEP_ONLY") and name not in os.environ["SWEEP_ONLY"].split(","):
             continue
+        if fn == "ax_e":  # N/4 elements: G is 6 fields
+            Na = N // 4
+            G = bc.fill(torch.empty((Na, 6, P1, P1, P1), dtype=torch.float64, device="cuda"), 11)
+            Ua, Wa = U[:Na], V[:Na]
+            fn = lambda: bc.ax_e(D, Ua, G, out=Wa)  # noqa: E731
         ms = timeit(fn)
         res[name] = {"ms": round(ms, 4), "hbm_frac": round(by / ms / 1e6 / HBM, 3), "tflops": round(fl / ms / 1e9, 2)}
     print(json.dumps({"lib": os.path.basename(bc.LIB_PATH), "p": p, "N": N, **res}), flush=True)
