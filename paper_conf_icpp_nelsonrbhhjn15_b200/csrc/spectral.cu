@@ -10,6 +10,13 @@
 // replacement); operator rows are read as 16-byte broadcast pairs, so every
 // shared-memory wavefront feeds 2R FMAs.  Intermediates never leave shared memory
 // (fusion); only U in and the outputs touch HBM.
+//
+// For odd P1 (smem layout == HBM layout) and batches of >= 128 elements the production
+// kernels are the warp-specialised TMA element rings further down (sumfact_tma_kernel,
+// local_grad3_tma_kernel, local_grad3_t_tma_kernel): a loader warp streams items of E
+// elements into an NB-slot ring with 1-D bulk copies, consumer groups run the same stages
+// (chunk_c) on their slot behind named barriers, and local_grad3's ur leaves through a
+// storer warp's bulk stores.
 #include <algorithm>
 #include <mutex>
 #include <type_traits>
