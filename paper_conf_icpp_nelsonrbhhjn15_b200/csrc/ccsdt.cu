@@ -502,7 +502,7 @@ __device__ __forceinline__ void tma_consume_stage(const unsigned char* A, const 
 
 // consumer: add a class's register tile into the accumulator cube at its permuted
 // positions (hp = storage positions of h1, h2, h3) and clear the registers
-template <int FE>
+template <int FE, bool STORE = false>
 __device__ __forceinline__ void tma_flush_class(double* acc_s, double (&c)[4][2][2], const int* hp, int warp, int gq,
                                                 int tq) {
     constexpr int CST = TmaGeo::CST;
@@ -531,13 +531,15 @@ __device__ __forceinline__ void tma_flush_class(double* acc_s, double (&c)[4][2]
 #pragma unroll
             for (int j = 0; j < 2; ++j) pos[mi][ni][j] = rowoff + (ni * 8 + permK(2 * tq + j)) * sb;
     }
+    // STORE: the unit's first class writes the cube (every position, out-of-range ones as
+    // zeros from the zero-filled operands) instead of read-modify-writing a zeroed cube
     double old[4][2][2];
 #pragma unroll
     for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
         for (int ni = 0; ni < 2; ++ni)
 #pragma unroll
-            for (int j = 0; j < 2; ++j) old[mi][ni][j] = acc_s[pos[mi][ni][j]];
+            for (int j = 0; j < 2; ++j) old[mi][ni][j] = STORE ? 0.0 : acc_s[pos[mi][ni][j]];
 #pragma unroll
     for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
@@ -1222,7 +1224,13 @@ struct TripMaps {
     CUtensorMap b[TRIP_MAXE];
 };
 
-__global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const __grid_constant__ TripParams P,
+#ifndef BC_F4_STORE_FIRST
+#define BC_F4_STORE_FIRST 1  // f4 16-cube: the first class stores into the cube (no zeroing pass)
+#endif
+#ifndef BC_F4_MINB
+#define BC_F4_MINB 2  // CTAs per SM of the 16-cube f4 kernel (1: ptxas took 130 registers)
+#endif
+__global__ void __launch_bounds__(TmaGeo::NT, BC_F4_MINB) ccsdt_triples_energy_kernel(const __grid_constant__ TripParams P,
                                                                           const __grid_constant__ TripMaps M,
                                                                           int units) {
     using TG = TmaGeo;
@@ -1326,14 +1334,19 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const 
             if (v < P.ns1) s1_issue(v, v, o, qv);
             cp_async_commit();
         }
-        for (int i = tid; i < BS * CST * CST; i += 256) acc_s[i] = 0.0;
-        named_bar_sync(1, 256);
+        if (nstage == 0 || !BC_F4_STORE_FIRST) {  // no d1/d2 class (s1 only): a zero cube
+            for (int i = tid; i < BS * CST * CST; i += 256) acc_s[i] = 0.0;
+            named_bar_sync(1, 256);
+        }
+        bool first_flush = BC_F4_STORE_FIRST;
         double c[4][2][2];
 #pragma unroll
         for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
             for (int ni = 0; ni < 2; ++ni) c[mi][ni][0] = c[mi][ni][1] = 0.0;
+        int cls_stages = 0;
         for (int st = 0; st < nstage; ++st, ++g) {
+            ++cls_stages;
             const int slot = g % NS;
             mbar_wait(bar_full + 8 * slot, (g / NS) & 1);
             const unsigned char* A = gbase + slot * TG::STAGE_BYTES;
@@ -1344,9 +1357,21 @@ __global__ void __launch_bounds__(TmaGeo::NT) ccsdt_triples_energy_kernel(const 
             else tma_consume_stage<FAM_D2>(A, B, P.smask[e], c, warp, gq, tq);
             release_slot(bar_empty + 8 * slot, lane);
             if (k0 + KC >= K && (e + 1 == P.nentry || P.ecls[e + 1] != P.ecls[e])) {
-                named_bar_sync(1, 256);  // no two classes flush concurrently (see ccsdt_tma_kernel)
-                if (d1) tma_flush_class<FAM_D1>(acc_s, c, P.hpos[P.ecls[e]], warp, gq, tq);
-                else tma_flush_class<FAM_D2>(acc_s, c, P.hpos[P.ecls[e]], warp, gq, tq);
+                // no two classes flush concurrently: the cube was zeroed behind a barrier, and
+                // a class spanning more than NS stages cannot overlap the previous class's
+                // flush (the producer refills a slot only after every consumer released it,
+                // so the fastest warp is at most NS stages ahead; as in ccsdt_tma_kernel)
+                if (BC_FLUSH_ALWAYS_BAR || cls_stages <= NS) named_bar_sync(1, 256);
+                cls_stages = 0;
+                const int* hp = P.hpos[P.ecls[e]];
+                if (first_flush) {  // the unit-start barrier ordered the previous unit's reads
+                    if (d1) tma_flush_class<FAM_D1, true>(acc_s, c, hp, warp, gq, tq);
+                    else tma_flush_class<FAM_D2, true>(acc_s, c, hp, warp, gq, tq);
+                    first_flush = false;
+                } else {
+                    if (d1) tma_flush_class<FAM_D1>(acc_s, c, hp, warp, gq, tq);
+                    else tma_flush_class<FAM_D2>(acc_s, c, hp, warp, gq, tq);
+                }
             }
         }
         // s1 rank-1 updates t3 += s t1[p4,h1] v2[h3,h2,p6,p5], accumulated in registers for
