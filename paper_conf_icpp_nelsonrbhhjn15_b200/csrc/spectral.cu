@@ -1091,8 +1091,8 @@ local_grad3_kernel(int64_t N, const double* __restrict__ D, const double* __rest
 #ifndef BC_L3_NUNR
 #define BC_L3_NUNR 1
 #endif
-#ifndef BC_L3_EAGER
-#define BC_L3_EAGER 1  // storer releases a slot as soon as its ur copy has read it
+#ifndef BC_L3_POLL
+#define BC_L3_POLL 1  // storer polls the slots (out-of-order items) instead of waiting in item order
 #endif
 template <int P1>
 using TmaLg3 = Ring<P1 * P1 * P1,
@@ -1125,9 +1125,9 @@ local_grad3_tma_kernel(int64_t N, const double* __restrict__ U, double* __restri
         if (lane == 0) ring_loader<TC>(N, U, slots, full0, empty0, nitems);
     } else if (warp == NG * NWG + 1) {
         if (lane == 0) {
-            for (int64_t j = 0; j < nitems; ++j) {
-                const int b = (int)(j % NB);
-                mbar_wait(done0 + 8 * b, (int)((j / NB) & 1));
+            // store item j (slot b) once its `done` phase completed, then release the slot as
+            // soon as the bulk copy has read it
+            auto store_item = [&](int64_t j, int b) {
                 const int64_t e0 = (blockIdx.x + j * gridDim.x) * E;
                 const int n = (int)imin64(E, N - e0) * NPTS;
                 const int h = item_lead(U + e0 * NPTS);  // == item_lead(ur + e0 * NPTS)
@@ -1138,14 +1138,36 @@ local_grad3_tma_kernel(int64_t N, const double* __restrict__ U, double* __restri
                 if (h + m < n) dst[n - 1] = in[n - 1];
                 if (m) bulk_store(dst + h, smem_u32(in + h), (uint32_t)m * 8u);
                 bulk_commit();
-                if constexpr (BC_L3_EAGER) {
-                    bulk_wait_read<0>();  // this item's copy has read its slot: release it now
-                    fence_proxy_async();
-                    mbar_arrive(empty0 + 8 * b);
-                } else if (j > 0) {
-                    bulk_wait_read<1>();  // item j-1's copy has read its slot
-                    fence_proxy_async();
-                    mbar_arrive(empty0 + 8 * (int)((j - 1) % NB));
+                bulk_wait_read<0>();
+                fence_proxy_async();
+                mbar_arrive(empty0 + 8 * b);
+            };
+            if constexpr (BC_L3_POLL) {
+                // slots are polled round robin (non-blocking test_wait), so an item finished
+                // by a fast group is stored and its slot released without waiting for an
+                // earlier item of a slower group (slot b holds items b, b + NB, ... in order,
+                // and its `done` barrier cannot run a phase ahead: the next phase needs this
+                // release)
+                int use[NB];
+#pragma unroll
+                for (int b = 0; b < NB; ++b) use[b] = 0;
+                int64_t left = nitems;
+                while (left > 0) {
+#pragma unroll
+                    for (int b = 0; b < NB; ++b) {
+                        const int64_t j = b + (int64_t)NB * use[b];
+                        if (j < nitems && mbar_test(done0 + 8 * b, use[b] & 1)) {
+                            store_item(j, b);
+                            ++use[b];
+                            --left;
+                        }
+                    }
+                }
+            } else {
+                for (int64_t j = 0; j < nitems; ++j) {
+                    const int b = (int)(j % NB);
+                    mbar_wait(done0 + 8 * b, (int)((j / NB) & 1));
+                    store_item(j, b);
                 }
             }
             bulk_wait<0>();
