@@ -141,6 +141,19 @@ int bc_ccsdt_d2_fused(const bc_tile_dims* d, double* t3, const double* const t2[
 int bc_ccsdt_s1_fused(const bc_tile_dims* d, double* t3, const double* const t1[9],
                       const double* const v2[9], void* stream);
 
+/* A fused family update followed by its check scalar (R18: the "CCSD(T) energy-style sum"
+ * the north star names for the checks; P:705-712 usage): family 1 = d1, 2 = d2, 3 = s1;
+ * a/b as bc_ccsdt_{d1,d2,s1}_fused.  After t3 += the listed variants,
+ *     ws[0] = E = bc_check_energy(d, t3, eps_h, eps_p) of the UPDATED t3
+ * (same definition and layouts; equal up to the order of the fp64 sum).  Where the 16-cube
+ * tensor-core kernel runs on full cubes (hole extents multiples of 16, equal hole and
+ * equal particle extents) the energy is accumulated in that kernel's t3 store pass (t3 is
+ * not read again); otherwise the update and a separate energy pass run back to back.
+ * ws: device, >= BC_CHECK_WS_DOUBLES doubles, not overlapping t3. */
+int bc_ccsdt_fused_energy(int family, const bc_tile_dims* d, double* t3, const double* const a[9],
+                          const double* const b[9], const double* eps_h, const double* eps_p,
+                          double* ws, void* stream);
+
 /* All 27 triples variants of one tile block fused, t3 never stored (
  * P:705-712 "representative of what executes at the socket level"):
  *     t3 = sum_v s1_v + sum_v d1_v + sum_v d2_v        (from zero, R3/R12/R23)

@@ -247,6 +247,27 @@ def ccsdt_fused(family: str, ext, t3: torch.Tensor, t2s, v2s) -> torch.Tensor:
     return t3
 
 
+def ccsdt_fused_energy(family: str, ext, t3: torch.Tensor, t2s, v2s, eps_h, eps_p, ws=None) -> torch.Tensor:
+    """t3 += the fused family (as ccsdt_fused), then ws[0] = check_energy of the updated t3
+    (fused into the tensor-core kernel's store pass where it runs on full cubes).
+    Returns ws[0] (device scalar)."""
+    fam = {"d1": 1, "d2": 2, "s1": 3}[family]
+    dev = t3.device
+    f = torch.float64
+    if ws is None:
+        ws = torch.empty(BC_CHECK_WS_DOUBLES, dtype=f, device=dev)
+    a, b = _ptr9(t2s, v2s, "t2", dev, *operand_sizes(family, ext))
+    d = _dims(ext)
+    h = int(ext[0]) + int(ext[1]) + int(ext[2])
+    pp = int(ext[3]) + int(ext[4]) + int(ext[5])
+    with _on(dev):
+        _check(lib.bc_ccsdt_fused_energy(fam, ctypes.byref(d), _dev(t3, f, "t3", dev, numel=_n3(ext)), a, b,
+                                         _dev(eps_h, f, "eps_h", dev, numel=h), _dev(eps_p, f, "eps_p", dev, numel=pp),
+                                         _dev(ws, f, "ws", dev, min_numel=BC_CHECK_WS_DOUBLES), _stream(t3)),
+               "bc_ccsdt_fused_energy")
+    return ws[0]
+
+
 def ccsdt_triples_energy(ext, s1, d1, d2, eps_h, eps_p, ws=None) -> torch.Tensor:
     """Energy of the t3 built from all (non-None) triples variants, t3 never stored.
     s1 = (t1s, v2s), d1 = (t2s, v2s), d2 = (t2s, v2s): lists of 9 (None = skip).

@@ -41,6 +41,7 @@ _SIGS = {
     "bc_ccsdt_d1_fused": [ctypes.POINTER(TileDims), _vp, PtrArray9, PtrArray9, _vp],
     "bc_ccsdt_d2_fused": [ctypes.POINTER(TileDims), _vp, PtrArray9, PtrArray9, _vp],
     "bc_ccsdt_s1_fused": [ctypes.POINTER(TileDims), _vp, PtrArray9, PtrArray9, _vp],
+    "bc_ccsdt_fused_energy": [_i32, ctypes.POINTER(TileDims), _vp, PtrArray9, PtrArray9, _vp, _vp, _vp, _vp],
     "bc_ccsdt_triples_energy": [ctypes.POINTER(TileDims), PtrArray9, PtrArray9, PtrArray9, PtrArray9, PtrArray9,
                                 PtrArray9, _vp, _vp, _vp, _vp],
     "bc_ccsdt_d1_tile": [_i32, _i32, _vp, _vp, _vp, _vp],

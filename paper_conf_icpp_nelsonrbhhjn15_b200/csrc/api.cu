@@ -17,7 +17,8 @@ int run_local_grad3(int64_t, int, const double*, const double*, double*, double*
 int run_local_grad3_t(int64_t, int, const double*, const double*, const double*, const double*, double*, cudaStream_t);
 int run_ax_e(int64_t, int, const double*, const double*, const double*, double*, cudaStream_t);
 int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const double* const* opA,
-              const double* const* opB, cudaStream_t s);
+              const double* const* opB, cudaStream_t s, const double* eps_h = nullptr, const double* eps_p = nullptr,
+              double* ws = nullptr);
 int run_sumfact3d_mma(int64_t, int, const double*, const double*, const double*, const double*, double*, double*,
                       cudaStream_t);
 int run_sumfact2d_mma(int64_t, int, const double*, const double*, const double*, double*, cudaStream_t);
@@ -126,8 +127,10 @@ static int ccsdt_one(int fam, int variant, const bc_tile_dims* d, double* t3, co
     return run_ccsdt(fam, e, t3, &variant, 1, &a, &b, as_stream(stream));
 }
 
+// eps_h/eps_p/ws non-null: also ws[0] = energy check of the updated t3 (bc_check_energy)
 static int ccsdt_fused(int fam, const bc_tile_dims* d, double* t3, const double* const* A,
-                       const double* const* B, void* stream) {
+                       const double* const* B, void* stream, const double* eps_h = nullptr,
+                       const double* eps_p = nullptr, double* ws = nullptr) {
     const bool needk = fam != 3;
     int st = check_dims(d, needk);
     if (st) return st;
@@ -138,6 +141,11 @@ static int ccsdt_fused(int fam, const bc_tile_dims* d, double* t3, const double*
     size_t na, nb;
     operand_elems(fam, e, &na, &nb);
     const size_t n3 = t3_elems(e);
+    if (ws) {
+        BC_REQUIRE(eps_h && eps_p, BC_ERR_ARG);
+        BC_REQUIRE(aligned(eps_h, 8) && aligned(eps_p, 8) && aligned(ws, 8), BC_ERR_ALIGN);
+        BC_REQUIRE(!overlap(ws, BC_CHECK_WS_DOUBLES * 8, t3, n3 * 8), BC_ERR_ALIAS);
+    }
     int vs[9], nv = 0;
     const double* pa[9];
     const double* pb[9];
@@ -151,13 +159,14 @@ static int ccsdt_fused(int fam, const bc_tile_dims* d, double* t3, const double*
         pb[nv] = B[v - 1];
         ++nv;
     }
-    if (nv == 0) return BC_OK;
+    if (nv == 0) return ws ? run_energy(e, t3, eps_h, eps_p, ws, as_stream(stream)) : BC_OK;
     const bool same_geometry = (e[0] == e[1] && e[1] == e[2] && e[3] == e[4] && e[4] == e[5]);
-    if (same_geometry) return run_ccsdt(fam, e, t3, vs, nv, pa, pb, as_stream(stream));
+    if (same_geometry) return run_ccsdt(fam, e, t3, vs, nv, pa, pb, as_stream(stream), eps_h, eps_p, ws);
     for (int t = 0; t < nv; ++t) {  // variants' t3 geometries differ: ascending single-variant passes
         st = run_ccsdt(fam, e, t3, &vs[t], 1, &pa[t], &pb[t], as_stream(stream));
         if (st) return st;
     }
+    if (ws) return run_energy(e, t3, eps_h, eps_p, ws, as_stream(stream));
     return BC_OK;
 }
 
@@ -285,6 +294,13 @@ int bc_ccsdt_d2_fused(const bc_tile_dims* d, double* t3, const double* const t2[
                       void* stream) {
     return ccsdt_fused(2, d, t3, t2, v2, stream);
 }
+int bc_ccsdt_fused_energy(int family, const bc_tile_dims* d, double* t3, const double* const a[9],
+                          const double* const b[9], const double* eps_h, const double* eps_p, double* ws,
+                          void* stream) {
+    BC_REQUIRE(family >= 1 && family <= 3 && ws != nullptr, BC_ERR_ARG);
+    return ccsdt_fused(family, d, t3, a, b, stream, eps_h, eps_p, ws);
+}
+
 int bc_ccsdt_s1_fused(const bc_tile_dims* d, double* t3, const double* const t1[9], const double* const v2[9],
                       void* stream) {
     return ccsdt_fused(3, d, t3, t1, v2, stream);

@@ -101,6 +101,11 @@ struct CcsdtParams {
     int ext[7];       // named extents h1 h2 h3 p4 p5 p6 k
     int qe[6];        // storage-position extents
     int ncube[3];     // cubes along q1, q2, q3
+    // optional energy check fused into the 16-cube TMA kernel's store pass (canonical
+    // storage only): ews[blockIdx.x] = sum over the stored t3 of t^2 / den (bc_check_energy)
+    const double* eps_h;
+    const double* eps_p;
+    double* ews;
 };
 
 // Per cube side BS: register tile TS (strided operand, one value per lane-stride) x TB
@@ -678,6 +683,7 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
         }
     };
     const bool full_cubes = P.qe[0] % BS == 0 && P.qe[1] % BS == 0 && P.qe[2] % BS == 0;
+    double energy = 0.0;  // fused energy check (P.ews; the launcher passes it for full cubes only)
     int g = 0;
     UnitDigits ud = unit_digits(blockIdx.x, rad);
     for (int u = blockIdx.x; u < units; u += gridDim.x) {
@@ -763,6 +769,28 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
             const int q0 = tid & 15, q1 = tid >> 4;
             double* dstg = P.t3 + pbase + (o[0] + q0) + (int64_t)Q0 * ((o[1] + q1) + (int64_t)P.qe[1] * o[2]);
             double* srcs = acc_s + q0 + CST * q1;
+            // fused energy check (canonical storage: q = h3, h2, h1, p6, p5, p4), the order
+            // of additions of bc_check_energy's denominator
+            double dh = 0.0, dp = 0.0;
+            const double* eh1 = P.eps_h;
+            if (P.ews) {
+                dh = P.eps_h[P.ext[N_H1] + P.ext[N_H2] + o[0] + q0] + P.eps_h[P.ext[N_H1] + o[1] + q1];
+                dp = P.eps_p[P.ext[N_P4] + P.ext[N_P5] + qv[0]];
+            }
+            const double dp5 = P.ews ? P.eps_p[P.ext[N_P4] + qv[1]] : 0.0, dp4 = P.ews ? P.eps_p[qv[2]] : 0.0;
+            // t^2 / den with a hardware reciprocal estimate refined by two Newton steps
+            // (relative error ~1 ulp; the DDIV sequence in the unit epilogue cost more than
+            // the separate energy pass it replaces)
+            auto en = [&](double t, int q2) {
+                if (P.ews) {
+                    const double den = (((dh + eh1[o[2] + q2]) - dp) - dp5) - dp4;
+                    double r;
+                    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(den));
+                    r = fma(r, fma(-den, r, 1.0), r);
+                    r = fma(r, fma(-den, r, 1.0), r);
+                    energy = fma(t * t, r, energy);
+                }
+            };
             const int un = u + gridDim.x;
             if (un < units) {
                 int on[3], lenn[3], qvn[3];
@@ -772,13 +800,19 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
                 const double* srcg = P.t3 + pbn + (on[0] + q0) + (int64_t)Q0 * ((on[1] + q1) + (int64_t)P.qe[1] * on[2]);
 #pragma unroll
                 for (int q2 = 0; q2 < BS; ++q2) {
-                    dstg[(int64_t)Q01 * q2] = srcs[CST * CST * q2];
+                    const double t = srcs[CST * CST * q2];
+                    dstg[(int64_t)Q01 * q2] = t;
                     cp_async_8_after_read(srcs + CST * CST * q2, srcg + (int64_t)Q01 * q2);
+                    en(t, q2);
                 }
                 cp_async_commit();
             } else {
 #pragma unroll
-                for (int q2 = 0; q2 < BS; ++q2) dstg[(int64_t)Q01 * q2] = srcs[CST * CST * q2];
+                for (int q2 = 0; q2 < BS; ++q2) {
+                    const double t = srcs[CST * CST * q2];
+                    dstg[(int64_t)Q01 * q2] = t;
+                    en(t, q2);
+                }
             }
         } else if (len[0] == BS && len[1] == BS && len[2] == BS) {
             const int q0 = tid & 15, q1 = tid >> 4;
@@ -796,6 +830,17 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
         }
     }
     cp_async_wait_all();
+    if (P.ews) {  // consumer-only block reduction (the producer warp has left)
+        __shared__ double red[TG::NCW];
+        for (int off = 16; off > 0; off >>= 1) energy += __shfl_xor_sync(0xffffffffu, energy, off);
+        if (lane == 0) red[warp] = energy;
+        named_bar_sync(1, 256);
+        if (tid == 0) {
+            double sum = 0.0;
+            for (int w = 0; w < TG::NCW; ++w) sum += red[w];
+            P.ews[blockIdx.x] = sum;
+        }
+    }
 }
 
 // ---- host: tensor maps (driver entry point, no -lcuda)
@@ -862,7 +907,7 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
         if (!ok) return 1;
     }
     const int64_t units = (int64_t)P.ncube[0] * P.ncube[1] * P.ncube[2] * P.qe[3] * P.qe[4] * P.qe[5];
-    if (units == 0) return BC_OK;
+    if (units == 0) return P.ews ? run_check_finalize(0, P.ews - 8, s) : BC_OK;
     auto go = [&](auto kern, size_t smem, int* occ) {
         if (*occ == 0) {
             cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -870,16 +915,19 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
             if (*occ < 1) *occ = 1;
         }
         const int64_t cap = (int64_t)num_sms() * *occ;
-        const int grid = (int)(units < cap ? units : cap);
+        int grid = (int)(units < cap ? units : cap);
+        if (P.ews && grid > CHECK_MAX_PARTIALS) grid = CHECK_MAX_PARTIALS;
         kern<<<grid, TmaGeo::NT, smem, s>>>(P, M, (int)units);
-        return launch_status();
+        const int st = launch_status();
+        if (st || !P.ews) return st;
+        return run_check_finalize(grid, P.ews - 8, s);  // ews = ws + 8: partials -> ws[0]
     };
     const size_t smem1 = 1024 + (size_t)TmaGeo::STAGE_BYTES + TmaGeo::ACC * 8 + 2 * 8;
     static PerDevice<int> occ_dev;
     int& occ = occ_dev.get();
     static PerDevice<int> occ1_dev;
     int& occ1 = occ1_dev.get();
-    if (P.nentry == 1 && BC_TC16_SINGLE_NS1) return go(ccsdt_tma_kernel<FAM, 1, 3>, smem1, &occ1);
+    if (P.nentry == 1 && BC_TC16_SINGLE_NS1 && !P.ews) return go(ccsdt_tma_kernel<FAM, 1, 3>, smem1, &occ1);
     return go(ccsdt_tma_kernel<FAM>, TmaGeo::SMEM, &occ);
 }
 
@@ -2440,8 +2488,25 @@ static int launch_ccsdt_bs(const CcsdtParams& P, cudaStream_t s) {
 }
 
 // Launch variants listed in `vs` (ascending), all sharing one t3 geometry.
+int run_energy(const int* ext7, const double* t3, const double* eh, const double* ep, double* ws, cudaStream_t s);
+static int run_ccsdt_impl(int fam, const int* ext7, double* t3, const int* vs, int nv, const double* const* opA,
+                          const double* const* opB, const double* eps_h, const double* eps_p, double* ws,
+                          bool* fused_energy, cudaStream_t s);
+
+// t3 += the listed variants; with ws != nullptr also ws[0] = the energy check of the updated
+// t3 (bc_check_energy), fused into the 16-cube TMA kernel's store pass where that kernel
+// runs on full cubes, else a separate pass after the update.
 int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const double* const* opA,
-              const double* const* opB, cudaStream_t s) {
+              const double* const* opB, cudaStream_t s, const double* eps_h, const double* eps_p, double* ws) {
+    bool fused = false;
+    const int st = run_ccsdt_impl(fam, ext7, t3, vs, nv, opA, opB, eps_h, eps_p, ws, &fused, s);
+    if (st || !ws || fused) return st;
+    return run_energy(ext7, t3, eps_h, eps_p, ws, s);
+}
+
+static int run_ccsdt_impl(int fam, const int* ext7, double* t3, const int* vs, int nv, const double* const* opA,
+                          const double* const* opB, const double* eps_h, const double* eps_p, double* ws,
+                          bool* fused_energy, cudaStream_t s) {
     CcsdtParams P{};
     P.t3 = t3;
     for (int q = 0; q < 7; ++q) P.ext[q] = ext7[q];
@@ -2501,8 +2566,22 @@ int run_ccsdt(int fam, const int* ext7, double* t3, const int* vs, int nv, const
     const int bs = tc_shape ? 16 : choose_bs(P.qe);
     for (int q = 0; q < 3; ++q) P.ncube[q] = (P.qe[q] + bs - 1) / bs;
     if (tc_shape) {
+        // the energy check rides along when every cube is full (its store pass covers t3)
+        const bool fuse = ws && P.qe[0] % 16 == 0 && P.qe[1] % 16 == 0 && P.qe[2] % 16 == 0 &&
+                          ext7[N_H1] == ext7[N_H2] && ext7[N_H2] == ext7[N_H3] && ext7[N_P4] == ext7[N_P5] &&
+                          ext7[N_P5] == ext7[N_P6];
+        if (fuse) {
+            P.eps_h = eps_h;
+            P.eps_p = eps_p;
+            P.ews = ws + 8;
+        }
         const int st = (fam == FAM_D1) ? launch_ccsdt_tma<FAM_D1>(P, s) : launch_ccsdt_tma<FAM_D2>(P, s);
-        if (st != 1) return st;
+        if (st != 1) {
+            *fused_energy = fuse;
+            return st;
+        }
+        P.eps_h = P.eps_p = nullptr;
+        P.ews = nullptr;
     }
 #define LAUNCH(F)                                                          \
     if (bs == 16) return launch_ccsdt_bs<F, 16>(P, s);                      \

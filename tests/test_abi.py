@@ -85,6 +85,12 @@ def test_ccsdt_validation(abi):
     assert L.bc_ccsdt_d1_tile(1, 0, FAKE, FAKE * 2, FAKE * 4, None) == -1
     empty = abi.PtrArray9()
     assert L.bc_ccsdt_d1_fused(ctypes.byref(d), FAKE, empty, empty, None) == 0  # nothing to do
+    # fused family + energy check: family range, ws required, eps required, ws must not alias t3
+    assert L.bc_ccsdt_fused_energy(0, ctypes.byref(d), FAKE, empty, empty, FAKE * 8, FAKE * 9, FAKE * 10, None) == -1
+    assert L.bc_ccsdt_fused_energy(4, ctypes.byref(d), FAKE, empty, empty, FAKE * 8, FAKE * 9, FAKE * 10, None) == -1
+    assert L.bc_ccsdt_fused_energy(2, ctypes.byref(d), FAKE, empty, empty, FAKE * 8, FAKE * 9, None, None) == -1
+    assert L.bc_ccsdt_fused_energy(2, ctypes.byref(d), FAKE, empty, empty, None, FAKE * 9, FAKE * 10, None) == -1
+    assert L.bc_ccsdt_fused_energy(2, ctypes.byref(d), FAKE, empty, empty, FAKE * 8, FAKE * 9, FAKE, None) == -3
 
 
 def test_python_binding_refuses_cpu_tensors(abi):

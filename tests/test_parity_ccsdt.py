@@ -131,6 +131,33 @@ def test_energy_check(bc):
     assert abs(got - ref) <= 1e-12 * abs(ref)
 
 
+@pytest.mark.parametrize("family", ["d1", "d2"])
+@pytest.mark.parametrize("ext", [(16,) * 7, (32, 32, 32, 2, 2, 2, 16), (20, 20, 20, 3, 3, 3, 12)])
+def test_fused_energy(bc, family, ext):
+    """bc_ccsdt_fused_energy: t3 += the fused family, ws[0] = energy check of the updated
+    t3.  Full 16-cubes take the energy fused into the tensor-core kernel's store pass
+    (tile 16; 32^3 holes = 8 cubes per plane); 20^3 holes (ragged cubes) run the separate
+    pass.  t3 bitwise equal to bc_ccsdt_*_fused; the energy equal to the oracle's energy of
+    the oracle-updated t3 within 1e-12 relative (the oracle: R18 definition)."""
+    na, nb = sizes(family, ext)
+    t3 = syn.tensor(10, (n3(ext),))
+    t2s = [syn.tensor(20 + v, (na,)) for v in range(1, 10)]
+    v2s = [syn.tensor(40 + v, (nb,)) for v in range(1, 10)]
+    eh = syn.tensor(60, (sum(ext[:3]),), kind=syn.KIND_RANGE, lo=-2.0, hi=-0.5)
+    ep = syn.tensor(61, (sum(ext[3:6]),), kind=syn.KIND_RANGE, lo=0.5, hi=2.0)
+    dt2, dv2 = [to_dev(x) for x in t2s], [to_dev(x) for x in v2s]
+    a3, b3 = to_dev(t3), to_dev(t3)
+    ws = torch.full((bc.BC_CHECK_WS_DOUBLES,), float("nan"), dtype=torch.float64, device="cuda")
+    bc.ccsdt_fused(family, ext, a3, dt2, dv2)
+    got = float(bc.ccsdt_fused_energy(family, ext, b3, dt2, dv2, to_dev(eh), to_dev(ep), ws).item())
+    assert torch.equal(a3, b3)
+    sep = float(bc.check_energy(ext, a3, to_dev(eh), to_dev(ep)).item())
+    ref_t3 = oracle.ccsdt_fused(family, ext, t3, t2s, v2s)
+    ref = oracle.energy(ext, ref_t3, eh, ep)
+    assert abs(got - ref) <= 1e-12 * abs(ref), (got, ref)
+    assert abs(got - sep) <= 1e-12 * abs(ref)
+
+
 # (24, ...) takes the exact-24-cube kernel (ccsdt_triples24_kernel): k = 8 (one chunk) and
 # k = 10 (a ragged second chunk, zero-filled by TMA)
 @pytest.mark.parametrize("ext", [(16,) * 7, (20, 20, 20, 4, 4, 4, 6), (24, 24, 24, 2, 2, 2, 8), (24, 24, 24, 2, 2, 2, 10)])
