@@ -730,6 +730,12 @@ int launch_sumfact3d_k(int64_t N, const T* A, const T* B, const T* C, const T* U
 #ifndef BC_T3_R
 #define BC_T3_R 3
 #endif
+#ifndef BC_T2_NUNR
+#define BC_T2_NUNR BC_CST_NUNROLL  // n-loop unroll of the 2-D ring's stages
+#endif
+#ifndef BC_T3_NUNR
+#define BC_T3_NUNR 4  // n-loop unroll of the 3-D ring's stages (P1 <= 5: full; measured)
+#endif
 #ifndef BC_T3S_NB
 #define BC_T3S_NB 10
 #endif
@@ -872,15 +878,18 @@ sumfact_tma_kernel(int64_t N, const double* __restrict__ U, double* __restrict__
             const int64_t e0 = (blockIdx.x + j * gridDim.x) * E;
             const int nlines = (int)imin64(E, N - e0) * NA * P1;
             double* in = slots + (size_t)b * TC::SLOT + item_lead(U + e0 * NPTS);
-            apply_lines_gc<P1, NA, 2, TC::R, NWG, C, 0, OUT_SMEM>(wg, in, in, nullptr, nullptr, nlines);
+            constexpr int U = NA == 1 ? BC_T2_NUNR : (P1 <= 5 ? P1 : BC_T3_NUNR);
+            apply_lines_gc<P1, NA, 2, TC::R, NWG, C, 0, OUT_SMEM, false, false, U>(wg, in, in, nullptr, nullptr, nlines);
             named_bar_sync(1 + grp, NWG * 32);
             if constexpr (NA == 1) {
-                apply_lines_gc<P1, 1, 1, TC::R, NWG, C, 1, OUT_GLOBAL>(wg, in, nullptr, nullptr, V + e0 * NPTS, nlines);
+                apply_lines_gc<P1, 1, 1, TC::R, NWG, C, 1, OUT_GLOBAL, false, false, U>(wg, in, nullptr, nullptr,
+                                                                                       V + e0 * NPTS, nlines);
             } else {
-                apply_lines_gc<P1, P1, 1, TC::R, NWG, C, 1, OUT_SMEM>(wg, in, in, nullptr, nullptr, nlines);
+                apply_lines_gc<P1, P1, 1, TC::R, NWG, C, 1, OUT_SMEM, false, false, U>(wg, in, in, nullptr, nullptr,
+                                                                                      nlines);
                 named_bar_sync(1 + grp, NWG * 32);
-                sq += apply_lines_gc<P1, P1, 0, TC::R, NWG, C, 2, OUT_GLOBAL, true>(wg, in, nullptr, nullptr,
-                                                                                      V + e0 * NPTS, nlines);
+                sq += apply_lines_gc<P1, P1, 0, TC::R, NWG, C, 2, OUT_GLOBAL, true, false, U>(wg, in, nullptr, nullptr,
+                                                                                             V + e0 * NPTS, nlines);
             }
             release_slot(empty0 + 8 * b, lane);
         }
@@ -1332,6 +1341,12 @@ local_grad3_t_kernel(int64_t N, const double* __restrict__ D, const double* __re
 #ifndef BC_LT_R
 #define BC_LT_R 3
 #endif
+#ifndef BC_LT_NUNR
+#define BC_LT_NUNR BC_CST_NUNROLL  // n-loop unroll of the local_grad3_t ring's stages
+#endif
+#ifndef BC_LT13_NUNR
+#define BC_LT13_NUNR 4  // ... at P1 = 13 (measured: 0.82-0.84 -> 0.85-0.86 of HBM; 4 is worse at p=4/8)
+#endif
 #ifndef BC_LT13_R
 #define BC_LT13_R 2  // P1 = 13: 169 lines on 3 warps x 64 lanes (R = 3 leaves one warp idle)
 #endif
@@ -1374,12 +1389,13 @@ local_grad3_t_tma_kernel(int64_t N, const double* __restrict__ ur, const double*
             double* bR = slot + item_lead(ur + gbase);
             double* bS = slot + TC::SUB + item_lead(us + gbase);
             double* bT = slot + 2 * TC::SUB + item_lead(ut + gbase);
-            apply_lines_gc<P1, P1, 2, TC::R, NWG, C, 0, OUT_SMEM, false, true>(wg, bR, bR, nullptr, nullptr, nlines);
+            constexpr int UN = P1 == 13 ? BC_LT13_NUNR : BC_LT_NUNR;
+            apply_lines_gc<P1, P1, 2, TC::R, NWG, C, 0, OUT_SMEM, false, true, UN>(wg, bR, bR, nullptr, nullptr, nlines);
             named_bar_sync(1 + grp, NWG * 32);
-            apply_lines_gc<P1, P1, 1, TC::R, NWG, C, 0, OUT_SMEM_ADD, false, true>(wg, bS, bS, bR, nullptr, nlines);
+            apply_lines_gc<P1, P1, 1, TC::R, NWG, C, 0, OUT_SMEM_ADD, false, true, UN>(wg, bS, bS, bR, nullptr, nlines);
             named_bar_sync(1 + grp, NWG * 32);
-            apply_lines_gc<P1, P1, 0, TC::R, NWG, C, 0, OUT_GLOBAL_ADD, false, true>(wg, bT, nullptr, bS, U + gbase,
-                                                                                     nlines);
+            apply_lines_gc<P1, P1, 0, TC::R, NWG, C, 0, OUT_GLOBAL_ADD, false, true, UN>(wg, bT, nullptr, bS, U + gbase,
+                                                                                         nlines);
             release_slot(empty0 + 8 * b, lane);
         }
     }
