@@ -583,7 +583,9 @@ __device__ __forceinline__ void unit_add(UnitDigits& x, const UnitDigits& s, con
         x.d[i] = carry ? v - r[i] : v;
     }
 }
-template <int FAM, int NSR = TmaGeo::NS, int MINB = BC_TC16_MINB>
+// EN: the fused energy check (a separate instantiation: the energy code in the store pass
+// slowed the plain kernel by 4-5% even when disabled at run time)
+template <int FAM, int NSR = TmaGeo::NS, int MINB = BC_TC16_MINB, bool EN = false>
 __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __grid_constant__ CcsdtParams P,
                                                                      const __grid_constant__ TmaMaps M, int units) {
     using TG = TmaGeo;
@@ -773,16 +775,18 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
             // of additions of bc_check_energy's denominator
             double dh = 0.0, dp = 0.0;
             const double* eh1 = P.eps_h;
-            if (P.ews) {
+            double dp5 = 0.0, dp4 = 0.0;
+            if constexpr (EN) {
                 dh = P.eps_h[P.ext[N_H1] + P.ext[N_H2] + o[0] + q0] + P.eps_h[P.ext[N_H1] + o[1] + q1];
                 dp = P.eps_p[P.ext[N_P4] + P.ext[N_P5] + qv[0]];
+                dp5 = P.eps_p[P.ext[N_P4] + qv[1]];
+                dp4 = P.eps_p[qv[2]];
             }
-            const double dp5 = P.ews ? P.eps_p[P.ext[N_P4] + qv[1]] : 0.0, dp4 = P.ews ? P.eps_p[qv[2]] : 0.0;
             // t^2 / den with a hardware reciprocal estimate refined by two Newton steps
             // (relative error ~1 ulp; the DDIV sequence in the unit epilogue cost more than
             // the separate energy pass it replaces)
             auto en = [&](double t, int q2) {
-                if (P.ews) {
+                if constexpr (EN) {
                     const double den = (((dh + eh1[o[2] + q2]) - dp) - dp5) - dp4;
                     double r;
                     asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(den));
@@ -830,7 +834,7 @@ __global__ void __launch_bounds__(TmaGeo::NT, MINB) ccsdt_tma_kernel(const __gri
         }
     }
     cp_async_wait_all();
-    if (P.ews) {  // consumer-only block reduction (the producer warp has left)
+    if constexpr (EN) {  // consumer-only block reduction (the producer warp has left)
         __shared__ double red[TG::NCW];
         for (int off = 16; off > 0; off >>= 1) energy += __shfl_xor_sync(0xffffffffu, energy, off);
         if (lane == 0) red[warp] = energy;
@@ -928,6 +932,10 @@ static int launch_ccsdt_tma(const CcsdtParams& P, cudaStream_t s) {
     static PerDevice<int> occ1_dev;
     int& occ1 = occ1_dev.get();
     if (P.nentry == 1 && BC_TC16_SINGLE_NS1 && !P.ews) return go(ccsdt_tma_kernel<FAM, 1, 3>, smem1, &occ1);
+    if (P.ews) {
+        static PerDevice<int> occe_dev;
+        return go(ccsdt_tma_kernel<FAM, TmaGeo::NS, BC_TC16_MINB, true>, TmaGeo::SMEM, &occe_dev.get());
+    }
     return go(ccsdt_tma_kernel<FAM>, TmaGeo::SMEM, &occ);
 }
 
