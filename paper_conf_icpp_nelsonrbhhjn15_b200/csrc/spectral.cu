@@ -1511,7 +1511,7 @@ ax_e_kernel(int64_t N, const double* __restrict__ D, const double* __restrict__ 
         __syncthreads();
         const int total = ne * G::NPTS;
         // G[e][c][q]: AXE_PB points per thread per batch, all 6*AXE_PB loads issued before use
-        constexpr int PB = AXE_PB;
+        constexpr int PB = P1 == 9 ? 8 : AXE_PB;  // measured: P1 = 9 0.57 -> 0.73 with 8; 8 is slower at 5 and 13
         for (int f0 = threadIdx.x; f0 < total; f0 += PB * NT) {
             T gv[PB][6];
 #pragma unroll

@@ -109,7 +109,7 @@ def test_local_grad3_t(bc, P1):
 
 
 @pytest.mark.parametrize("N", [7, 140])
-@pytest.mark.parametrize("P1", [2, 5, 8, 12, 13, 16])
+@pytest.mark.parametrize("P1", [2, 5, 8, 9, 12, 13, 16])
 def test_ax_e(bc, P1, N):
     D = syn.gll_derivative(P1 - 1)
     U = syn.tensor(1, (N, P1, P1, P1))
